@@ -1,0 +1,358 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 PROCLUS hot path (BASELINE.json metric).
+
+One step = one full PROCLUS clustering (init + iterative phase + refinement,
+Alg 1) of the C3 workload: n = 1,000,000 points x d = 15, k = 10, l = 5,
+A = 100, B = 10, minDev = 0.7, itrPat = 5 (PAPER.md P:370 defaults), on
+seeded synthetic data from the PROCLUS-style generator (synth/, P:374,
+P:386).  Each timed step uses a different run seed (the paper averages over
+runs).  value = clusterings / s over the whole job (max over ranks).
+
+  python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+
+N > 1 must be launched with torchrun (one process per GPU); rows are sharded
+across ranks and the k x d partial sums are combined with NCCL allreduce
+inside the library (strong scaling: the same 1M-point clustering).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+BASELINE_METRIC = "PROCLUS clusterings/sec (ms per run) at n=1M,d=15; HBM GB/s vs peak, 1/2/4/8 GPUs"
+UNIT = "clusterings/s"
+FALLBACK_HBM_GBS = 6650.0
+L2_FLUSH_BYTES = 256 << 20
+REF_SAMPLE_ROWS = 100_000
+
+
+def workload_config(args, n_gpus):
+    cfg = synth.CONFIGS[args.config]
+    return {
+        "workload": f"{args.config}: n={cfg['n']:,} d={cfg['d']} k={cfg['k']} l={cfg['l']} "
+                    f"A=100 B=10 minDev=0.7 itrPat=5, full-space metric {args.metric.upper()}",
+        "n": cfg["n"], "d": cfg["d"], "k": cfg["k"], "l": cfg["l"], "A": 100, "B": 10,
+        "minDev": 0.7, "itrPat": 5, "metric": args.metric.upper(),
+        "data_seed": args.data_seed, "run_seeds": f"{args.seed0}..{args.seed0 + args.steps - 1}",
+        "generator": f"{cfg['n_clusters']} Gaussian clusters in {cfg['subspace_dim']}-d subspaces, "
+                     "sd 5 on [0,100], 5% uniform noise, min-max normalised (P:374, P:386)",
+        "l2": "256 MiB L2 flush written between timed steps",
+        "parallelism": f"rows sharded over {n_gpus} GPU(s)" if n_gpus > 1 else "1 GPU",
+    }
+
+
+def read_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(kind):
+    """dram bytes per launch of `kind` from the committed ncu summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            j = json.load(f)
+        v = j.get(kind)
+        return None if v is None else float(v)
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "50", "-i", str(self.device)],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.out = ""
+        if self.proc is not None:
+            time.sleep(0.1)
+            self.proc.terminate()
+            try:
+                self.out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                self.out = ""
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in (self.out or "").strip().splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for name, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(name)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": mx, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def cpu_baseline_full(data, cfg, metric):
+    """The oracle as it stands: one full clustering of the workload, 1 core."""
+    import oracle
+
+    t = time.perf_counter()
+    r = oracle.proclus(data, cfg["k"], cfg["l"], seed=1, metric=metric)
+    dt = time.perf_counter() - t
+    return r, dt
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (this tier's reference arm)."""
+    import oracle
+
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    oracle.build()
+    data, cfg = synth.config_data(args.config, seed=args.data_seed)
+    ns = min(REF_SAMPLE_ROWS, cfg["n"])
+    sample = np.ascontiguousarray(data[:ns])
+    metric = 0 if args.metric == "l2" else 1
+    times = []
+    for s in range(args.warmup + args.steps):
+        t = time.perf_counter()
+        oracle.proclus(sample, cfg["k"], cfg["l"], seed=args.seed0 + s, metric=metric)
+        dt = time.perf_counter() - t
+        if s >= args.warmup:
+            times.append(dt)
+    mean = sum(times) / len(times)
+    value = (ns / cfg["n"]) / mean  # linear-in-n scaling of every pass
+    desc = (f"oracle (single-threaded fp64 C, -O2) on the first {ns:,} rows of the "
+            f"{args.config} dataset, one clustering per step (seeds {args.seed0}.."
+            f"{args.seed0 + args.steps - 1}), scaled to the full workload by n_sample/n")
+    line = {
+        "impl": "reference", "metric": BASELINE_METRIC, "value": value, "unit": UNIT,
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": mean * 1e3 * cfg["n"] / ns, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": workload_config(args, args.gpus),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_edbt_jorgensensape22_b200 as pk
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} needs torchrun with {args.gpus} processes "
+                         f"(WORLD_SIZE={world})")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    pk.lib()
+
+    data, cfg = synth.config_data(args.config, seed=args.data_seed)
+    n, d, k, l = cfg["n"], cfg["d"], cfg["k"], cfg["l"]
+    metric = pk.METRIC_L2 if args.metric == "l2" else pk.METRIC_L1
+    lo = n * rank // world
+    hi = n * (rank + 1) // world
+    shard = np.ascontiguousarray(data[lo:hi])
+    uid = None
+    if world > 1:
+        obj = [torch.cuda.nccl.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    stream = torch.cuda.Stream()
+    xdev = torch.from_numpy(shard).cuda()
+    labels = torch.empty(hi - lo, dtype=torch.int32, device="cuda")
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device="cuda")
+    common = dict(metric=metric, device=local, stream=stream.cuda_stream, world_size=world,
+                  rank=rank, n_global=n if world > 1 else 0, row_offset=lo if world > 1 else 0,
+                  nccl_unique_id=uid)
+    h = pk.Proclus(xdev, stats=True, **common)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+        torch.cuda.synchronize()
+
+    # warm-up
+    for s in range(args.warmup):
+        h.run(k, l, seed=args.seed0 + 1000 + s, labels=labels)
+    barrier()
+
+    agg = {}
+    step_ms = []
+    launches = 0
+    iters = []
+    with ClockSampler(local) as clk:
+        barrier()
+        for s in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.zero_()
+            ev0 = torch.cuda.Event(enable_timing=True)
+            ev1 = torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            r = h.run(k, l, seed=args.seed0 + s, labels=labels)
+            ev1.record(stream)
+            ev1.synchronize()
+            step_ms.append(ev0.elapsed_time(ev1))
+            iters.append(r.iterations)
+            st = h.stats()
+            launches += st["total_launches"]
+            for kind in pk.STAT_KINDS:
+                a = agg.setdefault(kind, dict(launches=0, ms=0.0, alg_bytes=0.0))
+                for f in ("launches", "ms", "alg_bytes"):
+                    a[f] += st[kind][f]
+        barrier()
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    value = args.steps / (total_ms / 1e3)
+
+    # dominant kernel (largest device time) and its roofline
+    passes = ["locality", "assign", "cost", "refine_x", "final", "greedy"]
+    dom = max(passes, key=lambda kk: agg[kk]["ms"])
+    a = agg[dom]
+    peak, peak_src = read_peak()
+    achieved = (a["alg_bytes"] / (a["ms"] / 1e3)) / 1e9 if a["ms"] > 0 and a["alg_bytes"] > 0 else None
+    kernels = {kk: {"launches": agg[kk]["launches"], "ms_total": round(agg[kk]["ms"], 4),
+                    "share": round(agg[kk]["ms"] / max(sum(v["ms"] for v in agg.values()), 1e-9), 4),
+                    "GBps": round(agg[kk]["alg_bytes"] / (agg[kk]["ms"] / 1e3) / 1e9, 1)
+                    if agg[kk]["ms"] > 0 and agg[kk]["alg_bytes"] > 0 else None}
+               for kk in pk.STAT_KINDS if agg[kk]["launches"] > 0}
+    roofline = {"bound": "hbm", "kernel": dom,
+                "achieved": round(achieved, 1) if achieved else None, "peak": peak,
+                "unit": "GB/s", "frac": round(achieved / peak, 4) if achieved else None,
+                "traffic": ncu_traffic(dom), "peak_source": peak_src,
+                "bytes_per_launch": a["alg_bytes"] / max(a["launches"], 1),
+                "model": "data 4nd + Dist rows 4n per active slot (locality); data 4nd + u8 "
+                         "labels n (assign, cost)"}
+
+    # end to end through the public API with host buffers: H2D of the step's
+    # data (pinned) + the whole run + D2H of labels / medoids / dims
+    e2e = None
+    if world == 1 and not args.no_e2e:
+        pinned = torch.from_numpy(shard).pin_memory()
+        hh = pk.Proclus(pinned.numpy(), metric=metric, device=local)
+        hlab = torch.empty(hi - lo, dtype=torch.int32).pin_memory()
+        e_steps = max(3, min(args.steps, 20))
+        for s in range(2):
+            hh.load(pinned.numpy())
+            hh.run(k, l, seed=args.seed0 + s, labels=hlab.numpy())
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for s in range(e_steps):
+            hh.load(pinned.numpy())
+            hh.run(k, l, seed=args.seed0 + s, labels=hlab.numpy())
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        hh.close()
+        e2e = {"value": e_steps / dt, "unit": UNIT, "steps": e_steps,
+               "h2d_bytes_per_step": int(shard.nbytes),
+               "d2h_bytes_per_step": int(4 * (hi - lo) + 8 * k + k * d)}
+
+    cpu = None
+    parity = None
+    if world == 1 and rank == 0 and not args.no_cpu_baseline:
+        import oracle
+
+        oracle.build()
+        o, dt = cpu_baseline_full(data, cfg, metric)
+        cpu = {"value": 1.0 / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"one full clustering of the {args.config} workload (seed 1) by the "
+                         f"single-threaded fp64 C oracle: {dt:.2f} s, {o.iterations} iterations"}
+        g = h.run(k, l, seed=1, labels=labels)
+        glab = labels.cpu().numpy()
+        parity = {"seed": 1, "labels_equal": bool(np.array_equal(glab, o.labels)),
+                  "medoids_equal": bool(np.array_equal(g.medoids, o.medoids)),
+                  "dims_equal": bool(np.array_equal(g.dims, o.dims)),
+                  "iterations": [g.iterations, o.iterations],
+                  "cost_rel_err": abs(g.cost - o.cost) / abs(o.cost)}
+    h.close()
+
+    if rank == 0:
+        clocks = clk.summary()
+        line = {
+            "metric": BASELINE_METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": total_ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic", "config": workload_config(args, world),
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches, "clocks": clocks,
+            "iterations_per_run": {"mean": sum(iters) / len(iters), "min": min(iters),
+                                   "max": max(iters)},
+            "kernels": kernels, "parity": parity,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier(device_ids=[local])
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", choices=["C1", "C2", "C3", "C4"], default="C3")
+    ap.add_argument("--metric", choices=["l2", "l1"], default="l2")
+    ap.add_argument("--data-seed", type=int, default=1)
+    ap.add_argument("--seed0", type=int, default=1)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3  # timing rule: at least 3 warm-up steps
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_gpu(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

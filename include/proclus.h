@@ -1,0 +1,196 @@
+/*
+ * proclus.h -- C ABI of the B200-native GPU-FAST-PROCLUS hot path.
+ *
+ * PROCLUS (Alg 1-6) as parallelised by GPU-FAST-PROCLUS
+ * (P:221-362), re-designed for sm_100a.  Citations are to
+ * /root/reference/PAPER.md line numbers (P:<n>); readings of garbled or
+ * silent passages are listed in DESIGN.md section 3 and tagged [Rn].
+ *
+ * Problem statement (Alg 1 header P:107): given Data in R^{n x d}, the
+ * number of clusters k, the average number of dimensions l, the sample
+ * constants A, B, the bad-medoid threshold minDev and the patience itrPat,
+ * return k disjoint clusters C, their subspaces D and medoids M.
+ *
+ * Conventions shared by every entry point:
+ *  - Every function returns a proclus_status.  On a non-OK status the
+ *    contents of output buffers are unspecified and proclus_last_error()
+ *    returns a message describing the cause (thread-local, valid until the
+ *    next call on the same thread).
+ *  - Input data is row-major (point-major) n x d fp32.  Values must be finite.
+ *  - A handle owns all device memory it allocates (data copy, the Dist cache
+ *    of P:153, H of eq 5, labels, partial sums).  It is not thread-safe: one
+ *    call at a time per handle.  Distinct handles are independent.
+ *  - Determinism: identical (data, parameters, seed, device type) give
+ *    bit-identical outputs.
+ *  - Randomness (P:241 leaves it unspecified) follows reading R2: SplitMix64
+ *    streams keyed by (seed, k) for the sample / greedy start and by
+ *    (seed, k, l) for MCur and the replacement draws.
+ */
+#ifndef PROCLUS_H
+#define PROCLUS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define PROCLUS_API __attribute__((visibility("default")))
+#else
+#define PROCLUS_API
+#endif
+
+#define PROCLUS_ABI_VERSION 1
+#define PROCLUS_K_MAX 32   /* k <= 32: per-point medoid bitmasks are 32-bit */
+#define PROCLUS_D_MAX 1024
+
+typedef struct proclus_handle proclus_handle;
+
+typedef enum {
+  PROCLUS_OK = 0,
+  PROCLUS_EINVAL = -1,    /* argument outside the documented domain       */
+  PROCLUS_ENOMEM = -2,    /* host or device allocation failed             */
+  PROCLUS_ECUDA = -3,     /* a CUDA runtime call failed                   */
+  PROCLUS_ENCCL = -4,     /* a NCCL call failed (world_size > 1)          */
+  PROCLUS_EINTERNAL = -5  /* invariant violated inside the library        */
+} proclus_status;
+
+/* Full-space metric of Greedy (Alg 2 l.4) and ComputeL (Alg 3 l.3).
+ * The paper uses Euclidean distance; north_star names
+ * L1.  Reading R1: one option for both steps, L2 by default. */
+typedef enum { PROCLUS_METRIC_L2 = 0, PROCLUS_METRIC_L1 = 1 } proclus_metric;
+
+typedef struct {
+  int32_t device;          /* CUDA device ordinal; -1 = current device      */
+  int32_t metric;          /* proclus_metric                                */
+  int32_t max_iter;        /* cap on iterative-phase iterations; <=0: 10000 */
+  int32_t data_on_device;  /* 1: `data` passed to create/load is a device
+                              pointer (row-major n x d fp32) on `device`    */
+  void* stream;            /* cudaStream_t to run on; NULL: handle-owned    */
+  int32_t trace;           /* 1: record a per-iteration trace (see below)   */
+  /* Row-sharded multi-GPU (one process per GPU, P:235 data parallelism
+   * extended across GPUs).  world_size 1 = single GPU.  With world_size > 1
+   * this rank owns rows [row_offset, row_offset + n) of an n_global-row
+   * dataset and every k x d partial sum is combined by ncclAllReduce. */
+  int32_t world_size;
+  int32_t rank;
+  int64_t n_global;        /* 0: = n                                         */
+  int64_t row_offset;
+  const void* nccl_unique_id;  /* 128-byte ncclUniqueId (world_size > 1)    */
+  int32_t stats;           /* 1: time every kernel launch with CUDA events on
+                              the handle's stream (see proclus_get_stats)   */
+} proclus_options;
+
+typedef struct {
+  int32_t* labels;      /* [n] caller-allocated (host, or device if
+                           labels_on_device): cluster id in [0,k), -1 for an
+                           outlier (RemoveOutliers).  With
+                           world_size > 1: this rank's n rows.               */
+  int64_t* medoids;     /* [k] caller-allocated host: row index (global) of
+                           the medoid of cluster i (MBest, P:134 [R16])      */
+  uint8_t* dims;        /* [k*d] caller-allocated host: dims[i*d+j] = 1 iff
+                           j is in D_i; k*l ones, >= 2 per row       */
+  double cost;          /* costBest of the iterative phase (eq 8/9 [R4])    */
+  int32_t iterations;   /* iterative-phase iterations executed              */
+  int32_t labels_on_device;  /* 1: `labels` is a device pointer             */
+} proclus_result;
+
+/* Per-iteration trace of the last proclus_run (options.trace = 1).  Each
+ * pointer may be NULL; arrays hold cap iterations (k or k*d per iteration).
+ * mcur are positions into M (the B*k potential medoids). */
+typedef struct {
+  int32_t cap;
+  int32_t count;        /* out: iterations recorded                         */
+  int32_t* mcur;        /* [cap*k]   */
+  double* delta;        /* [cap*k]   delta_i, Alg 3 l.4-7                  */
+  int64_t* nL;          /* [cap*k]   |L_i|                                 */
+  uint8_t* dims;        /* [cap*k*d] D                                     */
+  int64_t* sizes;       /* [cap*k]   |C_i|                                 */
+  double* cost;         /* [cap]                                           */
+  uint8_t* improved;    /* [cap]                                           */
+  uint8_t* bad;         /* [cap*k]   MBad                                  */
+  double* X;            /* [cap*k*d] X_ij                                  */
+} proclus_trace;
+
+/* Per-kernel measurements of the last proclus_run (options.stats = 1).
+ * kind order: pack, gather, greedy, prepare, locality, assign, cost,
+ * refine_x, final, split_tail.  Only launches that did work are counted
+ * (iterations enqueued speculatively after the device stopped return at
+ * once and are excluded).  alg_bytes follows the byte model of DESIGN.md
+ * section 6 (data bytes + Dist rows + labels; no padding, no partials). */
+#define PROCLUS_STAT_KINDS 10
+typedef struct {
+  int64_t launches[PROCLUS_STAT_KINDS];
+  double ms[PROCLUS_STAT_KINDS];         /* summed CUDA-event time          */
+  double alg_bytes[PROCLUS_STAT_KINDS];  /* algorithmic bytes moved          */
+  double run_ms;                         /* first to last event of the run  */
+  int64_t total_launches;                /* every kernel launch of the run  */
+} proclus_stats;
+
+/* Fill *opt with defaults (device -1, L2, max_iter 10000, host data, own
+ * stream, no trace, world_size 1). */
+PROCLUS_API proclus_status proclus_options_init(proclus_options* opt);
+
+/* Copy `data` (row-major n x d fp32) to the device in the library's layout.
+ * The caller keeps ownership of `data` and may free it on return.
+ * EINVAL: n < 1, d < 2 (sigma divides by d-1), d > PROCLUS_D_MAX,
+ * non-finite values, bad options. */
+PROCLUS_API proclus_status proclus_create(const float* data, int64_t n, int32_t d,
+                              proclus_handle** out);
+PROCLUS_API proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
+                                 const proclus_options* opt,
+                                 proclus_handle** out);
+
+/* Replace the handle's data with new values of the same shape (host or
+ * device pointer per the handle's options).  Drops all cached distances. */
+PROCLUS_API proclus_status proclus_load(proclus_handle* h, const float* data);
+
+/* One PROCLUS clustering (Alg 1): initialization (sample of A*k points,
+ * Greedy to B*k potential medoids), iterative phase (Alg 1
+ * l.5-14, with the FAST caches of section 3), refinement (Alg 1
+ * l.16-19).  #S = min(A*k, n), #M = min(B*k, #S) (clamped, not an error).
+ * EINVAL: k < 2, k > PROCLUS_K_MAX, l < 2, l > d, A < 1, B < 1, #M < k,
+ * minDev <= 0 or not finite, itrPat < 1, out == NULL or missing arrays. */
+PROCLUS_API proclus_status proclus_run(proclus_handle* h, int32_t k, int32_t l, int32_t A,
+                           int32_t B, double minDev, int32_t itrPat,
+                           uint64_t seed, proclus_result* out);
+
+/* Multiple parameter settings over the grid ks x ls (k outer,
+ * l inner; outs has nk*nl entries, each with its own arrays).
+ * reuse_level 1: every setting equals an independent proclus_run(k, l, seed)
+ *   ("multi-param 1": the Dist cache and H are reused between settings that
+ *   share M, i.e. the same k).
+ * reuse_level 2: S and M are drawn once for k_max (greedy once) and
+ *   Dist, H, delta', |L| are reused across the whole grid ("multi-param 2").
+ * EINVAL: reuse_level not in {1,2}, empty grid, any invalid (k, l). */
+PROCLUS_API proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks,
+                                 int32_t nk, const int32_t* ls, int32_t nl,
+                                 int32_t A, int32_t B, double minDev,
+                                 int32_t itrPat, uint64_t seed,
+                                 int32_t reuse_level, proclus_result* outs);
+
+/* Copy the trace of the last run (requires options.trace = 1). */
+PROCLUS_API proclus_status proclus_get_trace(proclus_handle* h, proclus_trace* tr);
+
+/* Copy the per-kernel measurements of the last run (options.stats = 1). */
+PROCLUS_API proclus_status proclus_get_stats(proclus_handle* h, proclus_stats* st);
+
+/* Number of kernel launches issued by the last run (for the bench's
+ * gpu_launches). */
+PROCLUS_API int64_t proclus_last_launches(proclus_handle* h);
+
+/* NULL-safe; waits for outstanding work, frees everything the handle owns. */
+PROCLUS_API void proclus_destroy(proclus_handle* h);
+
+/* Thread-local description of the last failure on this thread. */
+PROCLUS_API const char* proclus_last_error(void);
+
+/* Library / ABI version and the sm architecture the kernels target (100). */
+PROCLUS_API int32_t proclus_abi_version(void);
+PROCLUS_API int32_t proclus_target_sm(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PROCLUS_H */

@@ -1,0 +1,746 @@
+// proclus_api.cu -- the C ABI of include/proclus.h and the host driver of
+// the B200 PROCLUS hot path.  The host only draws the sample (Alg 1 l.2) and
+// the initial MCur, allocates everything up front and launches; the
+// iterative phase (Alg 1 l.5-14) including its control runs on the device.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/proclus.h"
+#include "proclus_kernels.h"
+
+using namespace pc;
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+
+static proclus_status fail(proclus_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define CK(call)                                                              \
+  do {                                                                        \
+    cudaError_t e_ = (call);                                                  \
+    if (e_ != cudaSuccess)                                                    \
+      return fail(PROCLUS_ECUDA, "%s failed: %s (%s:%d)", #call,              \
+                  cudaGetErrorString(e_), __FILE__, __LINE__);                \
+  } while (0)
+
+#define CKN(call)                                                             \
+  do {                                                                        \
+    ncclResult_t r_ = (call);                                                 \
+    if (r_ != ncclSuccess)                                                    \
+      return fail(PROCLUS_ENCCL, "%s failed: %s", #call,                      \
+                  ncclGetErrorString(r_));                                    \
+  } while (0)
+
+#define TRY(expr)                                                             \
+  do {                                                                        \
+    proclus_status s_ = (expr);                                               \
+    if (s_ != PROCLUS_OK) return s_;                                          \
+  } while (0)
+
+// ------------------------------------------------------------------ RNG
+// SplitMix64 streams (reading R2).  Host side of the library; the oracle has
+// its own independent implementation.
+static uint64_t sm_next(uint64_t* s) {
+  uint64_t z = (*s += 0x9E3779B97F4A7C15ULL);
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+static uint64_t sm_uniform(uint64_t* s, uint64_t m) {
+  return (uint64_t)(((unsigned __int128)sm_next(s) * m) >> 64);
+}
+static uint64_t sm_once(uint64_t x) { return sm_next(&x); }
+static uint64_t stream_sm(uint64_t seed, int64_t k_sm) {
+  return sm_once(sm_once(seed) + (uint64_t)k_sm);
+}
+static uint64_t stream_it(uint64_t seed, int64_t k, int64_t l) {
+  return sm_once(sm_once(sm_once(seed) + (uint64_t)k) + (uint64_t)l + 4294967296ULL);
+}
+
+// ------------------------------------------------------------------ handle
+template <class T>
+struct DBuf {
+  T* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t count) {
+    if (count <= cap && p) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    cudaError_t e = cudaMalloc(&p, sizeof(T) * (count ? count : 1));
+    if (e == cudaSuccess) cap = count;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+struct proclus_handle {
+  int dev = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int64_t n = 0, n_pad = 0, n_total = 0, row_offset = 0;
+  int d = 0;
+  int metric = 0, max_iter = 10000;
+  bool data_on_device = false, trace = false;
+  int world = 1, rank = 0;
+  ncclComm_t comm = nullptr;
+  int num_sms = 148;
+  int64_t launches = 0;
+
+  DBuf<float> xs, staging;
+  DBuf<int> flag;
+  // init-phase products
+  DBuf<long long> sids, mids;
+  DBuf<float> srows, mrows;
+  DBuf<int> spos;
+  DBuf<double> pickdist;
+  std::vector<int64_t> h_mids;
+  int64_t nS = 0, nM = 0;
+  bool m_valid = false;
+  uint64_t m_seed = 0;
+  int m_ksm = 0, m_A = 0, m_B = 0;
+  // caches of GPU-FAST-PROCLUS (persist across settings of run_multi)
+  DBuf<float> dist;
+  DBuf<double> H, dprev;
+  DBuf<long long> nL;
+  DBuf<unsigned char> found, used;
+  // per-run buffers
+  DBuf<unsigned char> lab;
+  DBuf<double> med, X, Z, mu, part, red, Delta;
+  DBuf<int> dlist, pool, out_labels;
+  DBuf<unsigned char> dmask;
+  DBuf<long long> partc, redc;
+  DBuf<DevState> st;
+  DevState* h_st = nullptr;  // pinned
+  // trace
+  int tr_cap = 0;
+  DBuf<int> t_mcur;
+  DBuf<double> t_delta, t_cost, t_X;
+  DBuf<long long> t_nL, t_sizes;
+  DBuf<unsigned char> t_dims, t_improved, t_bad;
+  int last_k = 0, tr_count = 0;
+  // per-launch CUDA events (options.stats)
+  bool stats = false;
+  struct Rec {
+    int kind, iter;
+    cudaEvent_t a, b;
+  };
+  std::vector<cudaEvent_t> evpool;
+  size_t evnext = 0;
+  std::vector<Rec> recs;
+  size_t rec_done = 0;
+  proclus_stats last_stats{};
+};
+
+enum Kind {
+  K_PACK = 0, K_GATHER, K_GREEDY, K_PREPARE, K_LOC, K_ASG, K_COST, K_REF, K_FIN, K_SPLIT
+};
+
+static cudaEvent_t ev_get(proclus_handle* h) {
+  if (h->evnext == h->evpool.size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    h->evpool.push_back(e);
+  }
+  return h->evpool[h->evnext++];
+}
+
+// Launch `f` on the handle's stream, bracketed by events when stats are on.
+template <class F>
+static void launch(proclus_handle* h, int kind, int iter, F&& f) {
+  h->launches += 1;
+  if (!h->stats) {
+    f();
+    return;
+  }
+  cudaEvent_t a = ev_get(h), b = ev_get(h);
+  cudaEventRecord(a, h->stream);
+  f();
+  cudaEventRecord(b, h->stream);
+  h->recs.push_back({kind, iter, a, b});
+}
+
+static proclus_status set_device(proclus_handle* h) {
+  CK(cudaSetDevice(h->dev));
+  return PROCLUS_OK;
+}
+
+extern "C" {
+
+const char* proclus_last_error(void) { return g_err.c_str(); }
+int32_t proclus_abi_version(void) { return PROCLUS_ABI_VERSION; }
+int32_t proclus_target_sm(void) { return 100; }
+
+proclus_status proclus_options_init(proclus_options* opt) {
+  if (!opt) return fail(PROCLUS_EINVAL, "opt is NULL");
+  memset(opt, 0, sizeof(*opt));
+  opt->device = -1;
+  opt->metric = PROCLUS_METRIC_L2;
+  opt->max_iter = 10000;
+  opt->world_size = 1;
+  return PROCLUS_OK;
+}
+
+static proclus_status upload_data(proclus_handle* h, const float* data) {
+  const size_t bytes = sizeof(float) * (size_t)h->n * h->d;
+  const float* src = data;
+  if (!h->data_on_device) {
+    CK(h->staging.ensure((size_t)h->n * h->d));
+    CK(cudaMemcpyAsync(h->staging.p, data, bytes, cudaMemcpyHostToDevice, h->stream));
+    src = h->staging.p;
+  }
+  CK(cudaMemsetAsync(h->flag.p, 0, sizeof(int), h->stream));
+  launch(h, K_PACK, -1, [&] {
+    launch_pack_soa(src, h->n, h->d, h->n_pad, h->xs.p, h->flag.p, h->stream);
+  });
+  CK(cudaGetLastError());
+  int bad = 0;
+  CK(cudaMemcpyAsync(&bad, h->flag.p, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  if (bad) return fail(PROCLUS_EINVAL, "data contains non-finite values");
+  h->m_valid = false;  // cached M / Dist rows refer to old data
+  return PROCLUS_OK;
+}
+
+proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
+                                 const proclus_options* opt, proclus_handle** out) {
+  if (!out) return fail(PROCLUS_EINVAL, "out is NULL");
+  *out = nullptr;
+  proclus_options o;
+  if (opt)
+    o = *opt;
+  else
+    proclus_options_init(&o);
+  if (!data) return fail(PROCLUS_EINVAL, "data is NULL");
+  if (n < 1) return fail(PROCLUS_EINVAL, "n must be >= 1 (got %lld)", (long long)n);
+  if (d < 2 || d > PROCLUS_D_MAX)
+    return fail(PROCLUS_EINVAL, "d must be in [2, %d] (got %d)", PROCLUS_D_MAX, d);
+  if (o.metric != PROCLUS_METRIC_L2 && o.metric != PROCLUS_METRIC_L1)
+    return fail(PROCLUS_EINVAL, "unknown metric %d", o.metric);
+  if (o.world_size < 1 || o.rank < 0 || o.rank >= o.world_size)
+    return fail(PROCLUS_EINVAL, "bad world_size/rank");
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  int dev = o.device;
+  if (dev < 0) CK(cudaGetDevice(&dev));
+  if (dev >= ndev) return fail(PROCLUS_EINVAL, "device %d >= device count %d", dev, ndev);
+  auto* h = new proclus_handle();
+  h->dev = dev;
+  h->n = n;
+  h->d = d;
+  h->n_pad = ((n + PMAX - 1) / PMAX) * PMAX;
+  h->n_total = o.n_global > 0 ? o.n_global : n;
+  h->row_offset = o.row_offset;
+  h->metric = o.metric;
+  h->max_iter = o.max_iter > 0 ? o.max_iter : 10000;
+  h->data_on_device = o.data_on_device != 0;
+  h->trace = o.trace != 0;
+  h->stats = o.stats != 0;
+  h->world = o.world_size;
+  h->rank = o.rank;
+  if (h->world == 1 && (h->n_total != n || h->row_offset != 0)) {
+    delete h;
+    return fail(PROCLUS_EINVAL, "n_global/row_offset need world_size > 1");
+  }
+  if (h->row_offset < 0 || h->row_offset + n > h->n_total) {
+    delete h;
+    return fail(PROCLUS_EINVAL, "shard [row_offset, row_offset+n) outside n_global");
+  }
+  proclus_status st = PROCLUS_OK;
+  auto cleanup = [&](proclus_status s) {
+    proclus_destroy(h);
+    return s;
+  };
+  if ((st = set_device(h)) != PROCLUS_OK) return cleanup(st);
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, dev) != cudaSuccess)
+    return cleanup(fail(PROCLUS_ECUDA, "cudaGetDeviceProperties failed"));
+  h->num_sms = prop.multiProcessorCount;
+  if (o.stream) {
+    h->stream = (cudaStream_t)o.stream;
+  } else {
+    if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess)
+      return cleanup(fail(PROCLUS_ECUDA, "cudaStreamCreate failed"));
+    h->own_stream = true;
+  }
+  if (h->world > 1) {
+    if (!o.nccl_unique_id) return cleanup(fail(PROCLUS_EINVAL, "nccl_unique_id required"));
+    ncclUniqueId id;
+    memcpy(&id, o.nccl_unique_id, sizeof(id));
+    ncclResult_t r = ncclCommInitRank(&h->comm, h->world, id, h->rank);
+    if (r != ncclSuccess)
+      return cleanup(fail(PROCLUS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
+  }
+  if (h->xs.ensure((size_t)h->n_pad * d) != cudaSuccess || h->flag.ensure(1) != cudaSuccess)
+    return cleanup(fail(PROCLUS_ENOMEM, "device allocation of %lld x %d failed",
+                        (long long)n, d));
+  if (cudaMallocHost(&h->h_st, sizeof(DevState)) != cudaSuccess)
+    return cleanup(fail(PROCLUS_ENOMEM, "pinned allocation failed"));
+  if ((st = upload_data(h, data)) != PROCLUS_OK) return cleanup(st);
+  *out = h;
+  return PROCLUS_OK;
+}
+
+proclus_status proclus_create(const float* data, int64_t n, int32_t d,
+                              proclus_handle** out) {
+  return proclus_create_ex(data, n, d, nullptr, out);
+}
+
+proclus_status proclus_load(proclus_handle* h, const float* data) {
+  if (!h || !data) return fail(PROCLUS_EINVAL, "NULL argument");
+  TRY(set_device(h));
+  return upload_data(h, data);
+}
+
+void proclus_destroy(proclus_handle* h) {
+  if (!h) return;
+  cudaSetDevice(h->dev);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  h->xs.release();
+  h->staging.release();
+  h->flag.release();
+  h->sids.release();
+  h->mids.release();
+  h->srows.release();
+  h->mrows.release();
+  h->spos.release();
+  h->pickdist.release();
+  h->dist.release();
+  h->H.release();
+  h->dprev.release();
+  h->nL.release();
+  h->found.release();
+  h->used.release();
+  h->lab.release();
+  h->med.release();
+  h->X.release();
+  h->Z.release();
+  h->mu.release();
+  h->part.release();
+  h->red.release();
+  h->Delta.release();
+  h->dlist.release();
+  h->pool.release();
+  h->out_labels.release();
+  h->dmask.release();
+  h->partc.release();
+  h->redc.release();
+  h->st.release();
+  h->t_mcur.release();
+  h->t_delta.release();
+  h->t_cost.release();
+  h->t_X.release();
+  h->t_nL.release();
+  h->t_sizes.release();
+  h->t_dims.release();
+  h->t_improved.release();
+  h->t_bad.release();
+  for (cudaEvent_t e : h->evpool) cudaEventDestroy(e);
+  if (h->h_st) cudaFreeHost(h->h_st);
+  if (h->comm) ncclCommDestroy(h->comm);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+}
+
+int64_t proclus_last_launches(proclus_handle* h) { return h ? h->launches : -1; }
+
+}  // extern "C"
+
+// ------------------------------------------------------------------ driver
+static proclus_status validate_setting(const proclus_handle* h, int k, int l, int A,
+                                       int B, double minDev, int itrPat) {
+  if (k < 2 || k > PROCLUS_K_MAX)
+    return fail(PROCLUS_EINVAL, "k must be in [2, %d] (got %d)", PROCLUS_K_MAX, k);
+  if (l < 2 || l > h->d) return fail(PROCLUS_EINVAL, "l must be in [2, d=%d] (got %d)", h->d, l);
+  if (A < 1 || B < 1) return fail(PROCLUS_EINVAL, "A and B must be >= 1");
+  if (!(minDev > 0.0) || !std::isfinite(minDev))
+    return fail(PROCLUS_EINVAL, "minDev must be finite and > 0");
+  if (itrPat < 1) return fail(PROCLUS_EINVAL, "itrPat must be >= 1");
+  int64_t nS = std::min<int64_t>((int64_t)A * k, h->n_total);
+  int64_t nM = std::min<int64_t>((int64_t)B * k, nS);
+  if (nM < k) return fail(PROCLUS_EINVAL, "#M = %lld < k = %d", (long long)nM, k);
+  return PROCLUS_OK;
+}
+
+static proclus_status allreduce(proclus_handle* h, void* buf, size_t count,
+                                ncclDataType_t t) {
+  if (h->world <= 1) return PROCLUS_OK;
+  CKN(ncclAllReduce(buf, buf, count, t, ncclSum, h->comm, h->stream));
+  return PROCLUS_OK;
+}
+
+static void reset_stats(proclus_handle* h) {
+  h->launches = 0;
+  h->evnext = 0;
+  h->recs.clear();
+  h->rec_done = 0;
+  memset(&h->last_stats, 0, sizeof(h->last_stats));
+}
+
+// Initialization phase (Alg 1 l.2-3): Data' by partial Fisher-Yates over
+// [0, n_total) (reading R13), Greedy on the GPU (Alg 2).  Keyed by
+// (seed, k_sm, A, B) so that run_multi can reuse it.
+static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint64_t seed) {
+  if (h->m_valid && h->m_seed == seed && h->m_ksm == k_sm && h->m_A == A && h->m_B == B)
+    return PROCLUS_OK;
+  const int64_t nS = std::min<int64_t>((int64_t)A * k_sm, h->n_total);
+  const int64_t nM = std::min<int64_t>((int64_t)B * k_sm, nS);
+  uint64_t st = stream_sm(seed, k_sm);
+  std::vector<long long> S((size_t)nS);
+  {
+    std::unordered_map<int64_t, int64_t> v;
+    v.reserve((size_t)(2 * nS + 1));
+    auto get = [&](int64_t i) {
+      auto it = v.find(i);
+      return it == v.end() ? i : it->second;
+    };
+    for (int64_t t = 0; t < nS; ++t) {
+      int64_t r = t + (int64_t)sm_uniform(&st, (uint64_t)(h->n_total - t));
+      int64_t vt = get(t), vr = get(r);
+      v[t] = vr;
+      v[r] = vt;
+      S[(size_t)t] = vr;
+    }
+  }
+  const int q0 = (int)sm_uniform(&st, (uint64_t)nS);
+  const int d = h->d;
+  CK(h->sids.ensure((size_t)nS));
+  CK(h->srows.ensure((size_t)nS * d));
+  CK(h->spos.ensure((size_t)nM));
+  CK(h->pickdist.ensure((size_t)nM));
+  CK(h->mrows.ensure((size_t)nM * d));
+  CK(h->mids.ensure((size_t)nM));
+  CK(cudaMemcpyAsync(h->sids.p, S.data(), sizeof(long long) * nS, cudaMemcpyHostToDevice,
+                     h->stream));
+  launch(h, K_GATHER, -1, [&] {
+    launch_gather_rows(h->xs.p, h->n_pad, d, h->sids.p, h->row_offset, h->n, (int)nS,
+                       h->srows.p, h->stream);
+  });
+  CK(cudaGetLastError());
+  TRY(allreduce(h, h->srows.p, (size_t)nS * d, ncclFloat));
+  cudaError_t ge = cudaSuccess;
+  launch(h, K_GREEDY, -1, [&] {
+    ge = launch_greedy(h->srows.p, (int)nS, d, (int)nM, q0, h->metric, h->spos.p,
+                       h->pickdist.p, h->stream);
+  });
+  CK(ge);
+  launch(h, K_GATHER, -1, [&] {
+    launch_gather_m(h->srows.p, h->sids.p, h->spos.p, (int)nM, d, h->mrows.p, h->mids.p,
+                    h->stream);
+  });
+  CK(cudaGetLastError());
+  h->h_mids.resize((size_t)nM);
+  CK(cudaMemcpyAsync(h->h_mids.data(), h->mids.p, sizeof(long long) * nM,
+                     cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  h->nS = nS;
+  h->nM = nM;
+  h->m_valid = true;
+  h->m_seed = seed;
+  h->m_ksm = k_sm;
+  h->m_A = A;
+  h->m_B = B;
+  // new M: the Dist / H caches (keyed by M position) start empty
+  CK(h->dist.ensure((size_t)nM * h->n_pad));
+  CK(h->H.ensure((size_t)nM * d));
+  CK(h->dprev.ensure((size_t)nM));
+  CK(h->nL.ensure((size_t)nM));
+  CK(h->found.ensure((size_t)nM));
+  CK(h->used.ensure((size_t)nM));
+  CK(cudaMemsetAsync(h->H.p, 0, sizeof(double) * nM * d, h->stream));
+  CK(cudaMemsetAsync(h->nL.p, 0, sizeof(long long) * nM, h->stream));
+  CK(cudaMemsetAsync(h->found.p, 0, nM, h->stream));
+  CK(cudaMemsetAsync(h->used.p, 0, nM, h->stream));
+  return PROCLUS_OK;
+}
+
+// Three-step tail for world_size > 1: reduce per-block partials, allreduce
+// the k x d vector over NVLink (NCCL), finalise on every rank.
+static proclus_status split_tail(proclus_handle* h, const RunParams& p, const PassShape& ps,
+                                 int tail, int iter) {
+  launch(h, K_SPLIT, iter, [&] { launch_reduce(p, ps, tail, h->stream); });
+  TRY(allreduce(h, p.red, (size_t)p.k * p.d, ncclFloat64));
+  TRY(allreduce(h, p.redc, KMAX, ncclInt64));
+  launch(h, K_SPLIT, iter, [&] { launch_tail(p, tail, h->stream); });
+  return PROCLUS_OK;
+}
+
+static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev,
+                                  int itrPat, uint64_t seed, proclus_result* out) {
+  const int d = h->d;
+  const int nM = (int)h->nM;
+  const PassShape ps = pass_shape(d, k, h->num_sms);
+  CK(configure_kernels(ps));
+  CK(h->lab.ensure((size_t)2 * h->n_pad));
+  CK(h->med.ensure((size_t)k * d));
+  CK(h->X.ensure((size_t)k * d));
+  CK(h->Z.ensure((size_t)k * d));
+  CK(h->mu.ensure((size_t)k * d));
+  CK(h->dlist.ensure((size_t)k * d));
+  CK(h->dmask.ensure((size_t)k * d));
+  CK(h->part.ensure((size_t)ps.grid * k * d));
+  CK(h->partc.ensure((size_t)ps.grid * KMAX));
+  CK(h->red.ensure((size_t)k * d));
+  CK(h->redc.ensure(KMAX));
+  CK(h->pool.ensure((size_t)nM));
+  CK(h->Delta.ensure(KMAX));
+  CK(h->st.ensure(1));
+  CK(h->out_labels.ensure((size_t)h->n));
+  if (h->trace) {
+    const int cap = std::min(h->max_iter, 4096);
+    h->tr_cap = cap;
+    CK(h->t_mcur.ensure((size_t)cap * k));
+    CK(h->t_delta.ensure((size_t)cap * k));
+    CK(h->t_nL.ensure((size_t)cap * k));
+    CK(h->t_sizes.ensure((size_t)cap * k));
+    CK(h->t_bad.ensure((size_t)cap * k));
+    CK(h->t_dims.ensure((size_t)cap * k * d));
+    CK(h->t_X.ensure((size_t)cap * k * d));
+    CK(h->t_cost.ensure((size_t)cap));
+    CK(h->t_improved.ensure((size_t)cap));
+  }
+  // initial MCur: k distinct positions of M (partial Fisher-Yates, stream IT)
+  uint64_t it = stream_it(seed, k, l);
+  std::vector<int> pool((size_t)nM);
+  for (int t = 0; t < nM; ++t) pool[(size_t)t] = t;
+  DevState& s = *h->h_st;
+  memset(&s, 0, sizeof(s));
+  for (int i = 0; i < k; ++i) {
+    int r = i + (int)sm_uniform(&it, (uint64_t)(nM - i));
+    std::swap(pool[(size_t)i], pool[(size_t)r]);
+    s.mcur[i] = pool[(size_t)i];
+    s.mbest[i] = pool[(size_t)i];
+  }
+  s.rng = it;
+  s.cost = 0.0;
+  s.cost_best = INFINITY;
+  s.cur_buf = 0;
+  s.best_buf = 1;
+  CK(cudaMemcpyAsync(h->st.p, &s, sizeof(DevState), cudaMemcpyHostToDevice, h->stream));
+
+  RunParams p;
+  memset(&p, 0, sizeof(p));
+  p.n = h->n;
+  p.n_pad = h->n_pad;
+  p.n_total = h->n_total;
+  p.d = d;
+  p.k = k;
+  p.l = l;
+  p.nM = nM;
+  p.itrPat = itrPat;
+  p.max_iter = h->max_iter;
+  p.metric = h->metric;
+  p.minDev = minDev;
+  p.xs = h->xs.p;
+  p.mrows = h->mrows.p;
+  p.dist = h->dist.p;
+  p.lab0 = h->lab.p;
+  p.lab1 = h->lab.p + h->n_pad;
+  p.H = h->H.p;
+  p.dprev = h->dprev.p;
+  p.nL = h->nL.p;
+  p.found = h->found.p;
+  p.used = h->used.p;
+  p.med = h->med.p;
+  p.dlist = h->dlist.p;
+  p.dmask = h->dmask.p;
+  p.X = h->X.p;
+  p.Z = h->Z.p;
+  p.mu = h->mu.p;
+  p.part = h->part.p;
+  p.partc = h->partc.p;
+  p.red = h->red.p;
+  p.redc = h->redc.p;
+  p.pool = h->pool.p;
+  p.st = h->st.p;
+  p.P = ps.P;
+  p.nchunks = (h->n + ps.P - 1) / ps.P;
+  p.fuse_tail = h->world == 1 ? 1 : 0;
+  p.out_labels = h->out_labels.p;
+  p.Delta = h->Delta.p;
+  if (h->trace) {
+    p.tr.cap = h->tr_cap;
+    p.tr.mcur = h->t_mcur.p;
+    p.tr.delta = h->t_delta.p;
+    p.tr.nL = h->t_nL.p;
+    p.tr.dims = h->t_dims.p;
+    p.tr.sizes = h->t_sizes.p;
+    p.tr.cost = h->t_cost.p;
+    p.tr.improved = h->t_improved.p;
+    p.tr.bad = h->t_bad.p;
+    p.tr.X = h->t_X.p;
+  }
+  if (out && out->labels_on_device && out->labels) p.out_labels = out->labels;
+
+  launch(h, K_PREPARE, -1, [&] { launch_prepare(p, h->stream); });
+  CK(cudaGetLastError());
+  // Iterative phase.  Kernels exit immediately once the device sets `done`,
+  // so iterations are enqueued speculatively in batches and the flag is read
+  // once per batch (the minimum run length is itrPat + 1).
+  int launched = 0;
+  int batch = itrPat + 1;
+  for (;;) {
+    for (int b = 0; b < batch; ++b) {
+      const int iter = launched + b;
+      launch(h, K_LOC, iter, [&] { launch_locality(p, ps, h->stream); });
+      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_LOC, iter));
+      launch(h, K_ASG, iter, [&] { launch_assign(p, ps, h->stream); });
+      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_ASG, iter));
+      launch(h, K_COST, iter, [&] { launch_cost(p, ps, h->stream); });
+      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_COST, iter));
+    }
+    CK(cudaGetLastError());
+    launched += batch;
+    CK(cudaMemcpyAsync(h->h_st, h->st.p, sizeof(DevState), cudaMemcpyDeviceToHost,
+                       h->stream));
+    CK(cudaStreamSynchronize(h->stream));
+    if (h->h_st->done) break;
+    if (launched >= h->max_iter) break;
+    batch = 2;
+  }
+  // Refinement phase (Alg 1 l.16-19)
+  launch(h, K_REF, -1, [&] { launch_refine_x(p, ps, h->stream); });
+  if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_REF, -1));
+  launch(h, K_FIN, -1, [&] { launch_final(p, ps, h->stream); });
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(h->h_st, h->st.p, sizeof(DevState), cudaMemcpyDeviceToHost, h->stream));
+  if (out) {
+    if (out->labels && !out->labels_on_device)
+      CK(cudaMemcpyAsync(out->labels, p.out_labels, sizeof(int32_t) * h->n,
+                         cudaMemcpyDeviceToHost, h->stream));
+    if (out->dims)
+      CK(cudaMemcpyAsync(out->dims, h->dmask.p, (size_t)k * d, cudaMemcpyDeviceToHost,
+                         h->stream));
+  }
+  CK(cudaStreamSynchronize(h->stream));
+  if (out) {
+    for (int i = 0; i < k; ++i)
+      if (out->medoids) out->medoids[i] = h->h_mids[(size_t)h->h_st->mbest[i]];
+    out->cost = h->h_st->cost_best;
+    out->iterations = h->h_st->iterations;
+  }
+  h->last_k = k;
+  h->tr_count = h->trace ? std::min(h->h_st->iterations, h->tr_cap) : 0;
+  if (h->stats) {
+    proclus_stats& S = h->last_stats;
+    const int T = h->h_st->iterations;
+    const double bytes_pass = 4.0 * (double)h->n * d + (double)h->n;  // data + u8 labels
+    float first = 0.f;
+    for (size_t r = h->rec_done; r < h->recs.size(); ++r) {
+      const auto& R = h->recs[r];
+      if (R.iter >= T) continue;  // speculative launch after the stop: no work
+      float ms = 0.f;
+      CK(cudaEventElapsedTime(&ms, R.a, R.b));
+      S.launches[R.kind] += 1;
+      S.ms[R.kind] += ms;
+      float from0 = 0.f;
+      CK(cudaEventElapsedTime(&from0, h->recs[0].a, R.b));
+      if (from0 > first) first = from0;
+    }
+    h->rec_done = h->recs.size();
+    if (first > S.run_ms) S.run_ms = first;
+    S.alg_bytes[K_LOC] += h->h_st->bytes_loc;
+    S.alg_bytes[K_ASG] += T * bytes_pass;
+    S.alg_bytes[K_COST] += T * bytes_pass;
+    S.alg_bytes[K_REF] += bytes_pass;
+    S.alg_bytes[K_FIN] += 4.0 * (double)h->n * d + 4.0 * (double)h->n;
+    S.total_launches = h->launches;
+  }
+  return PROCLUS_OK;
+}
+
+extern "C" {
+
+proclus_status proclus_run(proclus_handle* h, int32_t k, int32_t l, int32_t A, int32_t B,
+                           double minDev, int32_t itrPat, uint64_t seed,
+                           proclus_result* out) {
+  if (!h) return fail(PROCLUS_EINVAL, "handle is NULL");
+  if (!out || !out->medoids || !out->dims || !out->labels)
+    return fail(PROCLUS_EINVAL, "out and its labels/medoids/dims arrays are required");
+  TRY(validate_setting(h, k, l, A, B, minDev, itrPat));
+  TRY(set_device(h));
+  reset_stats(h);
+  TRY(init_phase(h, k, A, B, seed));
+  return run_setting(h, k, l, minDev, itrPat, seed, out);
+}
+
+proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks, int32_t nk,
+                                 const int32_t* ls, int32_t nl, int32_t A, int32_t B,
+                                 double minDev, int32_t itrPat, uint64_t seed,
+                                 int32_t reuse_level, proclus_result* outs) {
+  if (!h || !ks || !ls || !outs) return fail(PROCLUS_EINVAL, "NULL argument");
+  if (nk < 1 || nl < 1) return fail(PROCLUS_EINVAL, "empty parameter grid");
+  if (reuse_level != 1 && reuse_level != 2)
+    return fail(PROCLUS_EINVAL, "reuse_level must be 1 or 2 (3 is not implemented)");
+  int kmax = 0;
+  for (int a = 0; a < nk; ++a) {
+    kmax = std::max(kmax, ks[a]);
+    for (int b = 0; b < nl; ++b) {
+      TRY(validate_setting(h, ks[a], ls[b], A, B, minDev, itrPat));
+      proclus_result* o = &outs[a * nl + b];
+      if (!o->labels || !o->medoids || !o->dims)
+        return fail(PROCLUS_EINVAL, "outs[%d] arrays are required", a * nl + b);
+    }
+  }
+  TRY(set_device(h));
+  reset_stats(h);
+  if (reuse_level == 2) TRY(init_phase(h, kmax, A, B, seed));
+  for (int a = 0; a < nk; ++a)
+    for (int b = 0; b < nl; ++b) {
+      if (reuse_level == 1) TRY(init_phase(h, ks[a], A, B, seed));
+      TRY(run_setting(h, ks[a], ls[b], minDev, itrPat, seed, &outs[a * nl + b]));
+    }
+  return PROCLUS_OK;
+}
+
+proclus_status proclus_get_stats(proclus_handle* h, proclus_stats* st) {
+  if (!h || !st) return fail(PROCLUS_EINVAL, "NULL argument");
+  if (!h->stats) return fail(PROCLUS_EINVAL, "handle created without options.stats");
+  *st = h->last_stats;
+  return PROCLUS_OK;
+}
+
+proclus_status proclus_get_trace(proclus_handle* h, proclus_trace* tr) {
+  if (!h || !tr) return fail(PROCLUS_EINVAL, "NULL argument");
+  if (!h->trace) return fail(PROCLUS_EINVAL, "handle created without options.trace");
+  TRY(set_device(h));
+  const int c = std::min(tr->cap, h->tr_count);
+  const int k = h->last_k, d = h->d;
+  tr->count = c;
+  auto cp = [&](void* dst, const void* src, size_t bytes) -> proclus_status {
+    if (dst && bytes) CK(cudaMemcpy(dst, src, bytes, cudaMemcpyDeviceToHost));
+    return PROCLUS_OK;
+  };
+  TRY(cp(tr->mcur, h->t_mcur.p, sizeof(int) * c * k));
+  TRY(cp(tr->delta, h->t_delta.p, sizeof(double) * c * k));
+  TRY(cp(tr->nL, h->t_nL.p, sizeof(long long) * c * k));
+  TRY(cp(tr->dims, h->t_dims.p, (size_t)c * k * d));
+  TRY(cp(tr->sizes, h->t_sizes.p, sizeof(long long) * c * k));
+  TRY(cp(tr->cost, h->t_cost.p, sizeof(double) * c));
+  TRY(cp(tr->improved, h->t_improved.p, (size_t)c));
+  TRY(cp(tr->bad, h->t_bad.p, (size_t)c * k));
+  TRY(cp(tr->X, h->t_X.p, sizeof(double) * c * k * d));
+  return PROCLUS_OK;
+}
+
+}  // extern "C"

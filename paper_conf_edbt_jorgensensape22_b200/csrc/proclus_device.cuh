@@ -1,0 +1,138 @@
+// proclus_device.cuh -- device-side state, parameters and exact-arithmetic
+// helpers of the B200 PROCLUS hot path.  Citations: /root/reference/PAPER.md
+// line numbers (P:<n>); readings [Rn] are listed in DESIGN.md section 3.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace pc {
+
+constexpr int KMAX = 32;    // k <= 32: per-point medoid membership is a u32
+constexpr int WMAX = 8;     // warps per pass block (P <= 256)
+constexpr int PMAX = 256;   // points per streamed chunk
+
+// One medoid slot whose locality set changes in this iteration
+// (GPU-FAST-PROCLUS).  The band is (lo, hi]: Theorem 3.1 / eq 3.
+struct ActSlot {
+  int slot;      // cluster slot i in MCur
+  int mpos;      // MIdx_i: position in M, row of Dist and H
+  int compute;   // 1: DistFound is false -> compute and store Dist row
+  int lam;       // lambda_i (eq 6): +1 grow, -1 shrink
+  double lo, hi; // band (lo, hi]; lo = -inf on first use (L_i itself)
+  float lo32, hi32;  // round-to-nearest fp32 of lo / hi (cached-row test)
+};
+
+// Mutable control state of one run, resident in device memory so that the
+// whole iterative phase (Alg 1 l.5-14) is decided on the GPU.
+struct DevState {
+  unsigned long long rng;       // stream IT (reading R2), device copy
+  int mcur[KMAX];               // MCur as positions into M
+  int mbest[KMAX];              // MBest
+  long long sizes[KMAX];        // |C_i| of the current clustering
+  long long sizes_best[KMAX];   // |C_i| of CBest
+  double delta[KMAX];           // delta_i
+  double cost, cost_best;
+  int itr, iterations, done, cur_buf, best_buf, improved;
+  int n_act;
+  ActSlot act[KMAX];
+  int nD[KMAX];                 // |D_i|
+  unsigned int ticket[4];       // last-block tickets of the pass kernels
+  int err;
+  double bytes_loc;             // algorithmic bytes of the locality passes
+};
+
+struct TraceBufs {
+  int cap;
+  int* mcur;
+  double* delta;
+  long long* nL;
+  unsigned char* dims;
+  long long* sizes;
+  double* cost;
+  unsigned char* improved;
+  unsigned char* bad;
+  double* X;
+};
+
+struct RunParams {
+  long long n;        // rows on this device
+  long long n_pad;    // padded row count of the SoA layout (multiple of PMAX)
+  long long n_total;  // |Data| (all ranks): threshold of P:91 and eq 8
+  int d, k, l, nM, itrPat, max_iter, metric;
+  double minDev;
+  const float* xs;         // data, SoA [d][n_pad] fp32
+  const float* mrows;      // rows of M [nM][d] fp32
+  float* dist;             // Dist cache [nM][n_pad] fp32
+  unsigned char* lab0;     // label buffers (current / best, swapped by index)
+  unsigned char* lab1;
+  double* H;               // [nM][d] (eq 5)
+  double* dprev;           // [nM] delta' of the previous use
+  long long* nL;           // [nM] |L|
+  unsigned char* found;    // [nM] DistFound
+  unsigned char* used;     // [nM] delta' valid
+  double* med;             // [k][d] current (or best) medoid rows, fp64
+  int* dlist;              // [k][d] D_i as ascending dimension lists
+  unsigned char* dmask;    // [k][d]
+  double* X;               // [k][d]
+  double* Z;               // [k][d] scratch
+  double* mu;              // [k][d] centroid on D_i, index (i, t)
+  double* part;            // [grid][k*d] per-block partial sums
+  long long* partc;        // [grid][KMAX] per-block partial counts
+  double* red;             // [k*d] reduced sums (after allreduce)
+  long long* redc;         // [KMAX]
+  int* pool;               // [nM] scratch of the replacement step
+  DevState* st;
+  int P;                   // points per chunk == blockDim.x of pass kernels
+  long long nchunks;
+  int fuse_tail;           // 1: last block finalises (single GPU)
+  TraceBufs tr;
+  int* out_labels;         // final labels [n] int32 (refinement)
+  double* Delta;           // [k] outlier radii
+};
+
+// ---- exact fp64 arithmetic: explicit round-to-nearest intrinsics so that
+// nvcc never contracts into FMA; every expression below repeats the
+// oracle's evaluation order (ascending j, left-to-right).
+__device__ __forceinline__ double dadd(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ double dsub(double a, double b) { return __dsub_rn(a, b); }
+__device__ __forceinline__ double dmul(double a, double b) { return __dmul_rn(a, b); }
+__device__ __forceinline__ double ddiv(double a, double b) { return __ddiv_rn(a, b); }
+
+// Full-space distance ||p - q||: L2 = sqrt(sum_j (p_j - q_j)^2), L1
+// = sum_j |p_j - q_j|, j ascending.  p has stride ps, q stride 1.
+__device__ __forceinline__ double full_dist(const double* p, int ps,
+                                            const double* q, int d,
+                                            int metric) {
+  double s = 0.0;
+  if (metric == 1) {
+    for (int j = 0; j < d; ++j) s = dadd(s, fabs(dsub(p[j * ps], q[j])));
+    return s;
+  }
+  for (int j = 0; j < d; ++j) {
+    double t = dsub(p[j * ps], q[j]);
+    s = dadd(s, dmul(t, t));
+  }
+  return __dsqrt_rn(s);
+}
+
+// SplitMix64 (reading R2), the library's own device implementation.
+__device__ __forceinline__ unsigned long long sm64_next(unsigned long long* s) {
+  unsigned long long z = (*s += 0x9E3779B97F4A7C15ULL);
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+__device__ __forceinline__ unsigned long long sm64_uniform(unsigned long long* s,
+                                                           unsigned long long m) {
+  return __umul64hi(sm64_next(s), m);
+}
+
+// Order-preserving u64 key of a double (non-NaN); -0 is folded to +0 first.
+__device__ __forceinline__ unsigned long long sortable_key(double z) {
+  z = dadd(z, 0.0);
+  unsigned long long u = (unsigned long long)__double_as_longlong(z);
+  return (u >> 63) ? ~u : (u | 0x8000000000000000ULL);
+}
+
+}  // namespace pc

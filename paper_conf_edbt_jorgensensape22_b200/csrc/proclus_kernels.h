@@ -1,0 +1,55 @@
+// proclus_kernels.h -- host-side launchers of the sm_100a kernels
+// (implemented in proclus_kernels.cu, called by the C ABI in proclus_api.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "proclus_device.cuh"
+
+namespace pc {
+
+struct PassShape {
+  int P;          // points per chunk == threads per block
+  int grid;       // persistent blocks (multiple of the SM count)
+  size_t smem_loc, smem_asg, smem_cost, smem_ref, smem_fin;
+};
+
+// N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value.
+void launch_pack_soa(const float* in, long long n, int d, long long n_pad,
+                     float* xs, int* bad, cudaStream_t s);
+// rows of the given (global) ids; rows outside [row_offset, row_offset+n)
+// are zero (they are filled by another rank and summed by the allreduce).
+void launch_gather_rows(const float* xs, long long n_pad, int d,
+                        const long long* ids, long long row_offset,
+                        long long n_local, int cnt, float* out, cudaStream_t s);
+// Greedy (Alg 2) in one CTA: spos[nM] positions into S.
+cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0,
+                          int metric, int* spos, double* pickdist,
+                          cudaStream_t s);
+// M rows and ids from S rows and positions.
+void launch_gather_m(const float* srows, const long long* sids, const int* spos,
+                     int nM, int d, float* mrows, long long* mids,
+                     cudaStream_t s);
+
+PassShape pass_shape(int d, int k, int num_sms);
+cudaError_t configure_kernels(const PassShape& ps);
+
+// iteration prologue (delta, active slots) for the state's MCur
+void launch_prepare(const RunParams& p, cudaStream_t s);
+// the three passes of one iteration (Alg 3+4, Alg 5, Alg 6 + Alg 1 l.10-14)
+void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s);
+void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s);
+void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s);
+// refinement (Alg 1 l.16-19)
+void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s);
+void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s);
+
+// multi-GPU split tails: reduce per-block partials (1 block), and the
+// single-block finalisation after the host allreduce of red/redc.
+enum Tail { TAIL_LOC = 0, TAIL_ASG = 1, TAIL_COST = 2, TAIL_REF = 3 };
+void launch_reduce(const RunParams& p, const PassShape& ps, int tail,
+                   cudaStream_t s);
+void launch_tail(const RunParams& p, int tail, cudaStream_t s);
+
+}  // namespace pc

@@ -1,0 +1,216 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on
+the same seeded inputs and RNG streams.  Needs a B200 (``-m gpu``)."""
+import numpy as np
+import pytest
+
+import synth
+from parity import assert_parity
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def pk():
+    import torch
+
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    import paper_conf_edbt_jorgensensape22_b200 as pk
+
+    pk.lib()
+    return pk
+
+
+def run_both(pk, orc, data, k, l, *, A=100, B=10, minDev=0.7, itrPat=5, seed=1,
+             metric=0, trace=True):
+    with pk.Proclus(data, metric=metric, trace=trace) as h:
+        g = h.run(k, l, A, B, minDev, itrPat, seed)
+        gt = h.trace() if trace else None
+    o = orc.proclus(data, k, l, A, B, minDev, itrPat, seed, metric=metric, trace=trace)
+    return g, gt, o, o.trace if trace else None
+
+
+# ---------------------------------------------------------------- C1 sweep
+@pytest.mark.parametrize("seed", range(1, 41))
+def test_C1_seed_sweep(pk, orc, seed):
+    data, cfg = synth.config_data("C1", seed=seed)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
+    note = assert_parity(g, o, gt, ot, what=f"C1 seed {seed}")
+    if note:
+        pytest.skip(note)
+
+
+@pytest.mark.parametrize("seed", range(1, 9))
+def test_C1_L1_metric(pk, orc, seed):
+    data, cfg = synth.config_data("C1", seed=seed)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed, metric=1)
+    note = assert_parity(g, o, gt, ot, what=f"C1/L1 seed {seed}")
+    if note:
+        pytest.skip(note)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_C2(pk, orc, seed):
+    data, cfg = synth.config_data("C2", seed=seed)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
+    assert_parity(g, o, gt, ot, what=f"C2 seed {seed}")
+
+
+# ---------------------------------------------------------------- shapes / edges
+SHAPES = [
+    # n, d, k, l, A, B  (ragged n, several chunks, d around the warp size)
+    (1, 2, 2, 2, 100, 10),
+    (5, 3, 2, 2, 100, 10),
+    (257, 4, 3, 2, 100, 10),
+    (1000, 2, 4, 2, 50, 5),
+    (3001, 16, 6, 4, 30, 6),
+    (2049, 17, 5, 17, 40, 4),
+    (4097, 33, 8, 6, 20, 5),
+    (1500, 100, 10, 10, 20, 5),
+    (3000, 64, 32, 3, 8, 2),
+]
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_shapes(pk, orc, shape):
+    n, d, k, l, A, B = shape
+    if n < 2 * k:
+        data = np.random.default_rng(n).random((max(n, 1), d)).astype(np.float32)
+        if orc.validate(data, k, l, A, B) != 0:
+            with pytest.raises(pk.ProclusError):
+                pk.proclus(data, k, l, A, B)
+            return
+    data = synth.generate(n, d, max(2, k // 2), max(1, d // 3), seed=n)
+    g, gt, o, ot = run_both(pk, orc, data, k, l, A=A, B=B, seed=3)
+    assert_parity(g, o, gt, ot, what=f"shape {shape}")
+
+
+def test_duplicates_and_ties(pk, orc):
+    """Integer data with many duplicate points: delta_i = 0, exact distance
+    ties in greedy, in L_i membership and in the assignment argmin."""
+    rng = np.random.default_rng(7)
+    data = rng.integers(0, 4, size=(3000, 6)).astype(np.float32)
+    for seed in range(1, 6):
+        g, gt, o, ot = run_both(pk, orc, data, 6, 3, seed=seed)
+        assert_parity(g, o, gt, ot, what=f"ties seed {seed}")
+
+
+def test_constant_columns_and_identical_points(pk, orc):
+    data = synth.generate(2000, 8, 4, 3, seed=5)
+    data[:, 2] = 0.5
+    data[:, 5] = 0.25
+    g, gt, o, ot = run_both(pk, orc, data, 4, 3, seed=2)
+    assert_parity(g, o, gt, ot, what="constant columns")
+    same = np.tile(np.float32([0.1, 0.2, 0.3]), (500, 1))  # sigma = 0 everywhere
+    g, gt, o, ot = run_both(pk, orc, same, 3, 2, seed=1)
+    assert_parity(g, o, gt, ot, what="identical points")
+
+
+def test_clamped_M_and_full_shuffle(pk, orc):
+    data = synth.generate(400, 5, 3, 2, seed=8)
+    g, gt, o, ot = run_both(pk, orc, data, 4, 2, A=2, B=10, seed=4)  # #M = #S = 8
+    assert_parity(g, o, gt, ot, what="clamped")
+    g, gt, o, ot = run_both(pk, orc, data[:40], 4, 2, A=100, B=10, seed=4)  # #S = n
+    assert_parity(g, o, gt, ot, what="n == #S")
+
+
+def test_l_equals_d_and_l_2(pk, orc):
+    data = synth.generate(3000, 7, 4, 3, seed=9)
+    for l in (2, 7):
+        g, gt, o, ot = run_both(pk, orc, data, 5, l, seed=6)
+        assert_parity(g, o, gt, ot, what=f"l={l}")
+
+
+def test_itrPat_and_minDev_variants(pk, orc):
+    data, cfg = synth.config_data("C1", seed=11)
+    for itrPat, minDev in ((1, 0.7), (3, 0.1), (8, 1.5)):
+        g, gt, o, ot = run_both(pk, orc, data, 5, 3, itrPat=itrPat, minDev=minDev, seed=2)
+        assert_parity(g, o, gt, ot, what=f"itrPat={itrPat} minDev={minDev}")
+
+
+def test_max_iter_cap(pk, orc):
+    data, cfg = synth.config_data("C1", seed=3)
+    with pk.Proclus(data, max_iter=3) as h:
+        g = h.run(5, 3, seed=1)
+    o = orc.proclus(data, 5, 3, seed=1, max_iter=3)
+    assert g.iterations == 3
+    assert_parity(g, o, what="max_iter")
+
+
+def test_deterministic_and_handle_reuse(pk):
+    data, cfg = synth.config_data("C2", seed=4)
+    with pk.Proclus(data) as h:
+        a = h.run(10, 5, seed=3)
+        b = h.run(10, 5, seed=3)  # caches warm from the first run
+        c = h.run(10, 5, seed=4)
+    assert np.array_equal(a.labels, b.labels) and a.cost == b.cost
+    assert np.array_equal(a.medoids, b.medoids) and a.iterations == b.iterations
+    assert c.labels.shape == a.labels.shape
+
+
+def test_load_replaces_data(pk, orc):
+    d1, _ = synth.config_data("C1", seed=1)
+    d2, _ = synth.config_data("C1", seed=2)
+    with pk.Proclus(d1) as h:
+        h.run(5, 3, seed=1)
+        h.load(d2)
+        g = h.run(5, 3, seed=1)
+    assert_parity(g, orc.proclus(d2, 5, 3, seed=1), what="after load")
+
+
+def test_nonfinite_rejected(pk):
+    data = np.random.default_rng(0).random((100, 4)).astype(np.float32)
+    data[7, 1] = np.inf
+    with pytest.raises(pk.ProclusError) as e:
+        pk.Proclus(data)
+    assert e.value.status == pk.EINVAL
+
+
+def test_invalid_settings(pk):
+    data = synth.generate(300, 5, 3, 2, seed=1)
+    with pk.Proclus(data) as h:
+        for args in ((1, 3), (5, 1), (5, 6), (33, 2)):
+            with pytest.raises(pk.ProclusError):
+                h.run(*args)
+        with pytest.raises(pk.ProclusError):
+            h.run(5, 3, minDev=0.0)
+        with pytest.raises(pk.ProclusError):
+            h.run(5, 3, itrPat=0)
+        with pytest.raises(pk.ProclusError):
+            h.run(200, 3, A=1, B=1)  # #M = min(200, 300) ... k > K_MAX
+
+
+def test_device_resident_io(pk, orc):
+    import torch
+
+    data, cfg = synth.config_data("C1", seed=5)
+    xd = torch.from_numpy(data).cuda()
+    lab = torch.empty(data.shape[0], dtype=torch.int32, device="cuda")
+    with pk.Proclus(xd) as h:
+        g = h.run(5, 3, seed=5, labels=lab)
+    torch.cuda.synchronize()
+    g.labels = lab.cpu().numpy()
+    assert_parity(g, orc.proclus(data, 5, 3, seed=5), what="device io")
+
+
+# ---------------------------------------------------------------- multi-setting
+def test_run_multi_levels(pk, orc):
+    data = synth.generate(6000, 10, 5, 3, seed=12)
+    ks, ls = [3, 5], [2, 4]
+    for level in (1, 2):
+        with pk.Proclus(data) as h:
+            got = h.run_multi(ks, ls, seed=7, reuse_level=level)
+        want = orc.proclus_multi(data, ks, ls, seed=7, reuse_level=level)
+        for i, (g, o) in enumerate(zip(got, want)):
+            assert_parity(g, o, what=f"multi level {level} setting {i}")
+
+
+# ---------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("name,seed", [("C3", 1), ("C4", 1)])
+def test_full_size_configs(pk, orc, name, seed):
+    """BASELINE.json full sizes, in the bench's launch configuration: the
+    whole run against the oracle (seconds of CPU each)."""
+    data, cfg = synth.config_data(name, seed=seed)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
+    note = assert_parity(g, o, gt, ot, what=name)
+    if note:
+        pytest.skip(note)
