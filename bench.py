@@ -223,6 +223,7 @@ def run_gpu(args):
     barrier()
 
     agg = {}
+    tails, fallbacks = {}, {}
     step_ms = []
     launches = 0
     iters = []
@@ -241,6 +242,10 @@ def run_gpu(args):
             iters.append(r.iterations)
             st = h.stats()
             launches += st["total_launches"]
+            for kk, v in st["tail_ms"].items():
+                tails[kk] = tails.get(kk, 0.0) + v
+            for kk, v in st["fallbacks"].items():
+                fallbacks[kk] = fallbacks.get(kk, 0) + v
             for kind in pk.STAT_KINDS:
                 a = agg.setdefault(kind, dict(launches=0, ms=0.0, alg_bytes=0.0))
                 for f in ("launches", "ms", "alg_bytes"):
@@ -326,6 +331,8 @@ def run_gpu(args):
             "iterations_per_run": {"mean": sum(iters) / len(iters), "min": min(iters),
                                    "max": max(iters)},
             "kernels": kernels, "parity": parity,
+            "tails_ms_total": {kk: round(v, 4) for kk, v in tails.items()},
+            "exact_fallbacks": fallbacks,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -43,7 +43,7 @@ extern "C" {
 
 #define PROCLUS_ABI_VERSION 1
 #define PROCLUS_K_MAX 32   /* k <= 32: per-point medoid bitmasks are 32-bit */
-#define PROCLUS_D_MAX 1024
+#define PROCLUS_D_MAX 256  /* a 2-stage ring of 64-point chunks fits in SMEM */
 
 typedef struct proclus_handle proclus_handle;
 
@@ -126,6 +126,10 @@ typedef struct {
   double alg_bytes[PROCLUS_STAT_KINDS];  /* algorithmic bytes moved          */
   double run_ms;                         /* first to last event of the run  */
   int64_t total_launches;                /* every kernel launch of the run  */
+  double tail_ms[4];      /* single-block tails (locality, assign, cost,
+                             refine), device %globaltimer                  */
+  int64_t fallbacks[4];   /* exact fp64 re-decisions (locality, assign,
+                             final): points within the fp32 error bound    */
 } proclus_stats;
 
 /* Fill *opt with defaults (device -1, L2, max_iter 10000, host data, own

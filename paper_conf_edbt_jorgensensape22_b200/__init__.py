@@ -24,7 +24,7 @@ LIB_PATH = _build.LIB
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EINTERNAL = 0, -1, -2, -3, -4, -5
 METRIC_L2, METRIC_L1 = 0, 1
 K_MAX = 32
-D_MAX = 1024
+D_MAX = 256
 
 
 class ProclusError(RuntimeError):
@@ -48,7 +48,8 @@ STAT_KINDS = ["pack", "gather", "greedy", "prepare", "locality", "assign", "cost
 class proclus_stats(C.Structure):
     _fields_ = [("launches", C.c_int64 * 10), ("ms", C.c_double * 10),
                 ("alg_bytes", C.c_double * 10), ("run_ms", C.c_double),
-                ("total_launches", C.c_int64)]
+                ("total_launches", C.c_int64), ("tail_ms", C.c_double * 4),
+                ("fallbacks", C.c_int64 * 4)]
 
 
 class proclus_result(C.Structure):
@@ -314,6 +315,10 @@ class Proclus:
                for i, name in enumerate(STAT_KINDS)}
         out["run_ms"] = float(st.run_ms)
         out["total_launches"] = int(st.total_launches)
+        out["tail_ms"] = dict(zip(["locality", "assign", "cost", "refine_x"],
+                                  [float(v) for v in st.tail_ms]))
+        out["fallbacks"] = dict(zip(["locality", "assign", "final", "-"],
+                                    [int(v) for v in st.fallbacks]))
         return out
 
     @property

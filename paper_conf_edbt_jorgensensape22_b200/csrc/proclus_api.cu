@@ -1,13 +1,17 @@
 // proclus_api.cu -- the C ABI of include/proclus.h and the host driver of
 // the B200 PROCLUS hot path.  The host only draws the sample (Alg 1 l.2) and
 // the initial MCur, allocates everything up front and launches; the
-// iterative phase (Alg 1 l.5-14) including its control runs on the device.
+// iterative phase (Alg 1 l.5-14) including its control runs on the device,
+// by default as one CUDA graph whose while-node loops until the device-side
+// control clears the condition (no host round trip per iteration).
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <unordered_map>
@@ -94,6 +98,10 @@ struct DBuf {
   }
 };
 
+enum Kind {
+  K_PACK = 0, K_GATHER, K_GREEDY, K_PREPARE, K_LOC, K_ASG, K_COST, K_REF, K_FIN, K_SPLIT
+};
+
 struct proclus_handle {
   int dev = 0;
   cudaStream_t stream = nullptr;
@@ -101,7 +109,7 @@ struct proclus_handle {
   int64_t n = 0, n_pad = 0, n_total = 0, row_offset = 0;
   int d = 0;
   int metric = 0, max_iter = 10000;
-  bool data_on_device = false, trace = false;
+  bool data_on_device = false, trace = false, stats = false;
   int world = 1, rank = 0;
   ncclComm_t comm = nullptr;
   int num_sms = 148;
@@ -109,11 +117,13 @@ struct proclus_handle {
 
   DBuf<float> xs, staging;
   DBuf<int> flag;
+  DBuf<unsigned> colmax;
+  DBuf<double> scale, iscale;
   // init-phase products
   DBuf<long long> sids, mids;
   DBuf<float> srows, mrows;
   DBuf<int> spos;
-  DBuf<double> pickdist;
+  DBuf<double> pickdist, gscratch;
   std::vector<int64_t> h_mids;
   int64_t nS = 0, nM = 0;
   bool m_valid = false;
@@ -121,17 +131,23 @@ struct proclus_handle {
   int m_ksm = 0, m_A = 0, m_B = 0;
   // caches of GPU-FAST-PROCLUS (persist across settings of run_multi)
   DBuf<float> dist;
-  DBuf<double> H, dprev;
+  DBuf<long long> Hq;
+  DBuf<double> dprev;
   DBuf<long long> nL;
   DBuf<unsigned char> found, used;
   // per-run buffers
   DBuf<unsigned char> lab;
-  DBuf<double> med, X, Z, mu, part, red, Delta;
+  DBuf<double> med, X, Z, mu, Delta;
   DBuf<int> dlist, pool, out_labels;
   DBuf<unsigned char> dmask;
-  DBuf<long long> partc, redc;
+  DBuf<long long> accg, cntg;
   DBuf<DevState> st;
   DevState* h_st = nullptr;  // pinned
+  // graph of one run (prepare -> while{loc, asg, cost} -> refine, final)
+  cudaGraphExec_t gexec = nullptr;
+  RunParams gkey;
+  PassShape gshape;
+  bool gvalid = false;
   // trace
   int tr_cap = 0;
   DBuf<int> t_mcur;
@@ -140,7 +156,6 @@ struct proclus_handle {
   DBuf<unsigned char> t_dims, t_improved, t_bad;
   int last_k = 0, tr_count = 0;
   // per-launch CUDA events (options.stats)
-  bool stats = false;
   struct Rec {
     int kind, iter;
     cudaEvent_t a, b;
@@ -150,10 +165,6 @@ struct proclus_handle {
   std::vector<Rec> recs;
   size_t rec_done = 0;
   proclus_stats last_stats{};
-};
-
-enum Kind {
-  K_PACK = 0, K_GATHER, K_GREEDY, K_PREPARE, K_LOC, K_ASG, K_COST, K_REF, K_FIN, K_SPLIT
 };
 
 static cudaEvent_t ev_get(proclus_handle* h) {
@@ -185,6 +196,13 @@ static proclus_status set_device(proclus_handle* h) {
   return PROCLUS_OK;
 }
 
+static proclus_status allreduce(proclus_handle* h, void* buf, size_t count, ncclDataType_t t,
+                                ncclRedOp_t op = ncclSum) {
+  if (h->world <= 1) return PROCLUS_OK;
+  CKN(ncclAllReduce(buf, buf, count, t, op, h->comm, h->stream));
+  return PROCLUS_OK;
+}
+
 extern "C" {
 
 const char* proclus_last_error(void) { return g_err.c_str(); }
@@ -201,6 +219,11 @@ proclus_status proclus_options_init(proclus_options* opt) {
   return PROCLUS_OK;
 }
 
+}  // extern "C"
+
+// N0 pack + per-dimension fixed-point scales.  Cell sums of dimension j are
+// bounded by 2 * n_total * max|x_j| (|x - c| with c inside the column range,
+// or |x|), so e_j = 61 - ceil(log2(bound)) keeps every total below 2^61.
 static proclus_status upload_data(proclus_handle* h, const float* data) {
   const size_t bytes = sizeof(float) * (size_t)h->n * h->d;
   const float* src = data;
@@ -210,17 +233,43 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
     src = h->staging.p;
   }
   CK(cudaMemsetAsync(h->flag.p, 0, sizeof(int), h->stream));
+  CK(cudaMemsetAsync(h->colmax.p, 0, sizeof(unsigned) * h->d, h->stream));
   launch(h, K_PACK, -1, [&] {
-    launch_pack_soa(src, h->n, h->d, h->n_pad, h->xs.p, h->flag.p, h->stream);
+    launch_pack_soa(src, h->n, h->d, h->n_pad, h->xs.p, h->flag.p, h->colmax.p, h->stream);
   });
   CK(cudaGetLastError());
+  TRY(allreduce(h, h->colmax.p, h->d, ncclUint32, ncclMax));
+  TRY(allreduce(h, h->flag.p, 1, ncclInt32, ncclMax));
   int bad = 0;
+  std::vector<unsigned> cm((size_t)h->d);
   CK(cudaMemcpyAsync(&bad, h->flag.p, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(cm.data(), h->colmax.p, sizeof(unsigned) * h->d, cudaMemcpyDeviceToHost,
+                     h->stream));
   CK(cudaStreamSynchronize(h->stream));
   if (bad) return fail(PROCLUS_EINVAL, "data contains non-finite values");
+  std::vector<double> sc((size_t)h->d), isc((size_t)h->d);
+  for (int j = 0; j < h->d; ++j) {
+    float m;
+    memcpy(&m, &cm[(size_t)j], sizeof(float));
+    int e = 0;
+    if (m > 0.f) {
+      const double bound = 2.0 * (double)h->n_total * (double)m;
+      e = 61 - (int)std::ceil(std::log2(bound));
+      e = std::max(-1000, std::min(1000, e));
+    }
+    sc[(size_t)j] = std::ldexp(1.0, e);
+    isc[(size_t)j] = std::ldexp(1.0, -e);
+  }
+  CK(cudaMemcpyAsync(h->scale.p, sc.data(), sizeof(double) * h->d, cudaMemcpyHostToDevice,
+                     h->stream));
+  CK(cudaMemcpyAsync(h->iscale.p, isc.data(), sizeof(double) * h->d, cudaMemcpyHostToDevice,
+                     h->stream));
+  CK(cudaStreamSynchronize(h->stream));
   h->m_valid = false;  // cached M / Dist rows refer to old data
   return PROCLUS_OK;
 }
+
+extern "C" {
 
 proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
                                  const proclus_options* opt, proclus_handle** out) {
@@ -239,6 +288,12 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
     return fail(PROCLUS_EINVAL, "unknown metric %d", o.metric);
   if (o.world_size < 1 || o.rank < 0 || o.rank >= o.world_size)
     return fail(PROCLUS_EINVAL, "bad world_size/rank");
+  const int64_t n_total = o.n_global > 0 ? o.n_global : n;
+  if (o.world_size == 1 && (n_total != n || o.row_offset != 0))
+    return fail(PROCLUS_EINVAL, "n_global/row_offset need world_size > 1");
+  if (o.row_offset < 0 || o.row_offset + n > n_total)
+    return fail(PROCLUS_EINVAL, "shard [row_offset, row_offset+n) outside n_global");
+  if (n_total >= (int64_t)1 << 40) return fail(PROCLUS_EINVAL, "n_global too large");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
   int dev = o.device;
@@ -248,8 +303,8 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
   h->dev = dev;
   h->n = n;
   h->d = d;
-  h->n_pad = ((n + PMAX - 1) / PMAX) * PMAX;
-  h->n_total = o.n_global > 0 ? o.n_global : n;
+  h->n_pad = ((n + PAD_ALIGN - 1) / PAD_ALIGN) * PAD_ALIGN;
+  h->n_total = n_total;
   h->row_offset = o.row_offset;
   h->metric = o.metric;
   h->max_iter = o.max_iter > 0 ? o.max_iter : 10000;
@@ -258,14 +313,6 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
   h->stats = o.stats != 0;
   h->world = o.world_size;
   h->rank = o.rank;
-  if (h->world == 1 && (h->n_total != n || h->row_offset != 0)) {
-    delete h;
-    return fail(PROCLUS_EINVAL, "n_global/row_offset need world_size > 1");
-  }
-  if (h->row_offset < 0 || h->row_offset + n > h->n_total) {
-    delete h;
-    return fail(PROCLUS_EINVAL, "shard [row_offset, row_offset+n) outside n_global");
-  }
   proclus_status st = PROCLUS_OK;
   auto cleanup = [&](proclus_status s) {
     proclus_destroy(h);
@@ -291,9 +338,11 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
     if (r != ncclSuccess)
       return cleanup(fail(PROCLUS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
   }
-  if (h->xs.ensure((size_t)h->n_pad * d) != cudaSuccess || h->flag.ensure(1) != cudaSuccess)
-    return cleanup(fail(PROCLUS_ENOMEM, "device allocation of %lld x %d failed",
-                        (long long)n, d));
+  if (h->xs.ensure((size_t)h->n_pad * d) != cudaSuccess || h->flag.ensure(1) != cudaSuccess ||
+      h->colmax.ensure((size_t)d) != cudaSuccess || h->scale.ensure((size_t)d) != cudaSuccess ||
+      h->iscale.ensure((size_t)d) != cudaSuccess)
+    return cleanup(
+        fail(PROCLUS_ENOMEM, "device allocation of %lld x %d failed", (long long)n, d));
   if (cudaMallocHost(&h->h_st, sizeof(DevState)) != cudaSuccess)
     return cleanup(fail(PROCLUS_ENOMEM, "pinned allocation failed"));
   if ((st = upload_data(h, data)) != PROCLUS_OK) return cleanup(st);
@@ -301,8 +350,7 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
   return PROCLUS_OK;
 }
 
-proclus_status proclus_create(const float* data, int64_t n, int32_t d,
-                              proclus_handle** out) {
+proclus_status proclus_create(const float* data, int64_t n, int32_t d, proclus_handle** out) {
   return proclus_create_ex(data, n, d, nullptr, out);
 }
 
@@ -316,17 +364,22 @@ void proclus_destroy(proclus_handle* h) {
   if (!h) return;
   cudaSetDevice(h->dev);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->gexec) cudaGraphExecDestroy(h->gexec);
   h->xs.release();
   h->staging.release();
   h->flag.release();
+  h->colmax.release();
+  h->scale.release();
+  h->iscale.release();
   h->sids.release();
   h->mids.release();
   h->srows.release();
   h->mrows.release();
   h->spos.release();
   h->pickdist.release();
+  h->gscratch.release();
   h->dist.release();
-  h->H.release();
+  h->Hq.release();
   h->dprev.release();
   h->nL.release();
   h->found.release();
@@ -336,15 +389,13 @@ void proclus_destroy(proclus_handle* h) {
   h->X.release();
   h->Z.release();
   h->mu.release();
-  h->part.release();
-  h->red.release();
   h->Delta.release();
   h->dlist.release();
   h->pool.release();
   h->out_labels.release();
   h->dmask.release();
-  h->partc.release();
-  h->redc.release();
+  h->accg.release();
+  h->cntg.release();
   h->st.release();
   h->t_mcur.release();
   h->t_delta.release();
@@ -367,8 +418,8 @@ int64_t proclus_last_launches(proclus_handle* h) { return h ? h->launches : -1; 
 }  // extern "C"
 
 // ------------------------------------------------------------------ driver
-static proclus_status validate_setting(const proclus_handle* h, int k, int l, int A,
-                                       int B, double minDev, int itrPat) {
+static proclus_status validate_setting(const proclus_handle* h, int k, int l, int A, int B,
+                                       double minDev, int itrPat) {
   if (k < 2 || k > PROCLUS_K_MAX)
     return fail(PROCLUS_EINVAL, "k must be in [2, %d] (got %d)", PROCLUS_K_MAX, k);
   if (l < 2 || l > h->d) return fail(PROCLUS_EINVAL, "l must be in [2, d=%d] (got %d)", h->d, l);
@@ -379,13 +430,6 @@ static proclus_status validate_setting(const proclus_handle* h, int k, int l, in
   int64_t nS = std::min<int64_t>((int64_t)A * k, h->n_total);
   int64_t nM = std::min<int64_t>((int64_t)B * k, nS);
   if (nM < k) return fail(PROCLUS_EINVAL, "#M = %lld < k = %d", (long long)nM, k);
-  return PROCLUS_OK;
-}
-
-static proclus_status allreduce(proclus_handle* h, void* buf, size_t count,
-                                ncclDataType_t t) {
-  if (h->world <= 1) return PROCLUS_OK;
-  CKN(ncclAllReduce(buf, buf, count, t, ncclSum, h->comm, h->stream));
   return PROCLUS_OK;
 }
 
@@ -428,6 +472,7 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   CK(h->srows.ensure((size_t)nS * d));
   CK(h->spos.ensure((size_t)nM));
   CK(h->pickdist.ensure((size_t)nM));
+  CK(h->gscratch.ensure(greedy_scratch_doubles((int)nS)));
   CK(h->mrows.ensure((size_t)nM * d));
   CK(h->mids.ensure((size_t)nM));
   CK(cudaMemcpyAsync(h->sids.p, S.data(), sizeof(long long) * nS, cudaMemcpyHostToDevice,
@@ -440,8 +485,8 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   TRY(allreduce(h, h->srows.p, (size_t)nS * d, ncclFloat));
   cudaError_t ge = cudaSuccess;
   launch(h, K_GREEDY, -1, [&] {
-    ge = launch_greedy(h->srows.p, (int)nS, d, (int)nM, q0, h->metric, h->spos.p,
-                       h->pickdist.p, h->stream);
+    ge = launch_greedy(h->srows.p, (int)nS, d, (int)nM, q0, h->metric, h->gscratch.p,
+                       h->spos.p, h->pickdist.p, h->stream);
   });
   CK(ge);
   launch(h, K_GATHER, -1, [&] {
@@ -462,60 +507,116 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   h->m_B = B;
   // new M: the Dist / H caches (keyed by M position) start empty
   CK(h->dist.ensure((size_t)nM * h->n_pad));
-  CK(h->H.ensure((size_t)nM * d));
+  CK(h->Hq.ensure((size_t)nM * d));
   CK(h->dprev.ensure((size_t)nM));
   CK(h->nL.ensure((size_t)nM));
   CK(h->found.ensure((size_t)nM));
   CK(h->used.ensure((size_t)nM));
-  CK(cudaMemsetAsync(h->H.p, 0, sizeof(double) * nM * d, h->stream));
+  CK(cudaMemsetAsync(h->Hq.p, 0, sizeof(long long) * nM * d, h->stream));
   CK(cudaMemsetAsync(h->nL.p, 0, sizeof(long long) * nM, h->stream));
   CK(cudaMemsetAsync(h->found.p, 0, nM, h->stream));
   CK(cudaMemsetAsync(h->used.p, 0, nM, h->stream));
   return PROCLUS_OK;
 }
 
-// Three-step tail for world_size > 1: reduce per-block partials, allreduce
-// the k x d vector over NVLink (NCCL), finalise on every rank.
-static proclus_status split_tail(proclus_handle* h, const RunParams& p, const PassShape& ps,
-                                 int tail, int iter) {
-  launch(h, K_SPLIT, iter, [&] { launch_reduce(p, ps, tail, h->stream); });
-  TRY(allreduce(h, p.red, (size_t)p.k * p.d, ncclFloat64));
-  TRY(allreduce(h, p.redc, KMAX, ncclInt64));
+// world_size > 1: allreduce the fixed-point cell sums (exact in int64) over
+// NVLink (NCCL), then finalise on every rank.
+static proclus_status split_tail(proclus_handle* h, const RunParams& p, int tail, int iter) {
+  TRY(allreduce(h, p.accg, (size_t)p.k * p.d, ncclInt64));
+  TRY(allreduce(h, p.cntg, KMAX, ncclInt64));
   launch(h, K_SPLIT, iter, [&] { launch_tail(p, tail, h->stream); });
   return PROCLUS_OK;
 }
 
-static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev,
-                                  int itrPat, uint64_t seed, proclus_result* out) {
+// One run as a CUDA graph: prepare -> while(cond){locality, assign, cost} ->
+// refine_x -> final.  The cost tail sets the condition.  Rebuilt only when
+// the kernel parameters change (new buffers or setting).
+static proclus_status build_graph(proclus_handle* h, RunParams p, const PassShape& ps) {
+  if (h->gvalid && memcmp(&h->gkey, &p, sizeof(RunParams)) == 0 &&
+      memcmp(&h->gshape, &ps, sizeof(PassShape)) == 0)
+    return PROCLUS_OK;
+  if (h->gexec) {
+    cudaGraphExecDestroy(h->gexec);
+    h->gexec = nullptr;
+  }
+  h->gvalid = false;
+  const RunParams key = p;
+  cudaGraph_t g;
+  CK(cudaGraphCreate(&g, 0));
+  cudaGraphConditionalHandle cond;
+  CK(cudaGraphConditionalHandleCreate(&cond, g, 1, cudaGraphCondAssignDefault));
+  p.use_cond = 1;
+  p.cond = (unsigned long long)cond;
+  cudaStream_t cs;
+  CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  cudaGraph_t tmp;
+  // prepare
+  CK(cudaStreamBeginCaptureToGraph(cs, g, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+  launch_prepare(p, cs);
+  CK(cudaStreamEndCapture(cs, &tmp));
+  size_t nn = 0;
+  CK(cudaGraphGetNodes(g, nullptr, &nn));
+  std::vector<cudaGraphNode_t> nodes(nn);
+  CK(cudaGraphGetNodes(g, nodes.data(), &nn));
+  cudaGraphNode_t prep = nodes.back();
+  // while node
+  cudaGraphNodeParams cp = {};
+  cp.type = cudaGraphNodeTypeConditional;
+  cp.conditional.handle = cond;
+  cp.conditional.type = cudaGraphCondTypeWhile;
+  cp.conditional.size = 1;
+  cudaGraphNode_t wnode;
+  CK(cudaGraphAddNode(&wnode, g, &prep, 1, &cp));
+  cudaGraph_t body = cp.conditional.phGraph_out[0];
+  CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+  launch_locality(p, ps, cs);
+  launch_assign(p, ps, cs);
+  launch_cost(p, ps, cs);
+  CK(cudaStreamEndCapture(cs, &tmp));
+  // refinement after the loop
+  CK(cudaStreamBeginCaptureToGraph(cs, g, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
+  launch_refine_x(p, ps, cs);
+  launch_final(p, ps, cs);
+  CK(cudaStreamEndCapture(cs, &tmp));
+  CK(cudaStreamDestroy(cs));
+  cudaError_t e = cudaGraphInstantiate(&h->gexec, g, 0);
+  cudaGraphDestroy(g);
+  CK(e);
+  h->gkey = key;
+  h->gshape = ps;
+  h->gvalid = true;
+  return PROCLUS_OK;
+}
+
+static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev, int itrPat,
+                                  uint64_t seed, proclus_result* out) {
   const int d = h->d;
   const int nM = (int)h->nM;
   const PassShape ps = pass_shape(d, k, h->num_sms);
   CK(configure_kernels(ps));
   CK(h->lab.ensure((size_t)2 * h->n_pad));
-  CK(h->med.ensure((size_t)k * d));
-  CK(h->X.ensure((size_t)k * d));
-  CK(h->Z.ensure((size_t)k * d));
-  CK(h->mu.ensure((size_t)k * d));
-  CK(h->dlist.ensure((size_t)k * d));
-  CK(h->dmask.ensure((size_t)k * d));
-  CK(h->part.ensure((size_t)ps.grid * k * d));
-  CK(h->partc.ensure((size_t)ps.grid * KMAX));
-  CK(h->red.ensure((size_t)k * d));
-  CK(h->redc.ensure(KMAX));
-  CK(h->pool.ensure((size_t)nM));
+  CK(h->med.ensure((size_t)KMAX * d));
+  CK(h->X.ensure((size_t)KMAX * d));
+  CK(h->Z.ensure((size_t)KMAX * d));
+  CK(h->mu.ensure((size_t)KMAX * d));
+  CK(h->dlist.ensure((size_t)KMAX * d));
+  CK(h->dmask.ensure((size_t)KMAX * d));
+  CK(h->accg.ensure((size_t)NCOPY * KMAX * d));
+  CK(h->cntg.ensure((size_t)NCOPY * KMAX));
+  CK(h->pool.ensure((size_t)std::max<int64_t>(h->nM, 1024)));
   CK(h->Delta.ensure(KMAX));
   CK(h->st.ensure(1));
   CK(h->out_labels.ensure((size_t)h->n));
   if (h->trace) {
     const int cap = std::min(h->max_iter, 4096);
     h->tr_cap = cap;
-    CK(h->t_mcur.ensure((size_t)cap * k));
-    CK(h->t_delta.ensure((size_t)cap * k));
-    CK(h->t_nL.ensure((size_t)cap * k));
-    CK(h->t_sizes.ensure((size_t)cap * k));
-    CK(h->t_bad.ensure((size_t)cap * k));
-    CK(h->t_dims.ensure((size_t)cap * k * d));
-    CK(h->t_X.ensure((size_t)cap * k * d));
+    CK(h->t_mcur.ensure((size_t)cap * KMAX));
+    CK(h->t_delta.ensure((size_t)cap * KMAX));
+    CK(h->t_nL.ensure((size_t)cap * KMAX));
+    CK(h->t_sizes.ensure((size_t)cap * KMAX));
+    CK(h->t_bad.ensure((size_t)cap * KMAX));
+    CK(h->t_dims.ensure((size_t)cap * KMAX * d));
+    CK(h->t_X.ensure((size_t)cap * KMAX * d));
     CK(h->t_cost.ensure((size_t)cap));
     CK(h->t_improved.ensure((size_t)cap));
   }
@@ -532,11 +633,12 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
     s.mbest[i] = pool[(size_t)i];
   }
   s.rng = it;
-  s.cost = 0.0;
   s.cost_best = INFINITY;
   s.cur_buf = 0;
   s.best_buf = 1;
   CK(cudaMemcpyAsync(h->st.p, &s, sizeof(DevState), cudaMemcpyHostToDevice, h->stream));
+  CK(cudaMemsetAsync(h->accg.p, 0, sizeof(long long) * NCOPY * KMAX * d, h->stream));
+  CK(cudaMemsetAsync(h->cntg.p, 0, sizeof(long long) * NCOPY * KMAX, h->stream));
 
   RunParams p;
   memset(&p, 0, sizeof(p));
@@ -556,7 +658,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.dist = h->dist.p;
   p.lab0 = h->lab.p;
   p.lab1 = h->lab.p + h->n_pad;
-  p.H = h->H.p;
+  p.Hq = h->Hq.p;
   p.dprev = h->dprev.p;
   p.nL = h->nL.p;
   p.found = h->found.p;
@@ -567,13 +669,14 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.X = h->X.p;
   p.Z = h->Z.p;
   p.mu = h->mu.p;
-  p.part = h->part.p;
-  p.partc = h->partc.p;
-  p.red = h->red.p;
-  p.redc = h->redc.p;
+  p.accg = h->accg.p;
+  p.cntg = h->cntg.p;
+  p.scale = h->scale.p;
+  p.iscale = h->iscale.p;
   p.pool = h->pool.p;
   p.st = h->st.p;
   p.P = ps.P;
+  p.stages = ps.stages;
   p.nchunks = (h->n + ps.P - 1) / ps.P;
   p.fuse_tail = h->world == 1 ? 1 : 0;
   p.out_labels = h->out_labels.p;
@@ -592,37 +695,52 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   }
   if (out && out->labels_on_device && out->labels) p.out_labels = out->labels;
 
-  launch(h, K_PREPARE, -1, [&] { launch_prepare(p, h->stream); });
-  CK(cudaGetLastError());
-  // Iterative phase.  Kernels exit immediately once the device sets `done`,
-  // so iterations are enqueued speculatively in batches and the flag is read
-  // once per batch (the minimum run length is itrPat + 1).
-  int launched = 0;
-  int batch = itrPat + 1;
-  for (;;) {
-    for (int b = 0; b < batch; ++b) {
-      const int iter = launched + b;
-      launch(h, K_LOC, iter, [&] { launch_locality(p, ps, h->stream); });
-      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_LOC, iter));
-      launch(h, K_ASG, iter, [&] { launch_assign(p, ps, h->stream); });
-      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_ASG, iter));
-      launch(h, K_COST, iter, [&] { launch_cost(p, ps, h->stream); });
-      if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_COST, iter));
-    }
+  // graph mode unless per-launch events are wanted, multi-GPU (NCCL between
+  // kernels), or PROCLUS_GRAPH=0 (ncu cannot profile kernels of graphs that
+  // contain conditional nodes)
+  static const bool graph_env = [] {
+    const char* v = getenv("PROCLUS_GRAPH");
+    return !(v && v[0] == '0');
+  }();
+  const bool use_graph = h->world == 1 && !h->stats && graph_env;
+  if (use_graph) {
+    // one graph launch: the whole iterative + refinement phase on the device
+    TRY(build_graph(h, p, ps));
+    CK(cudaGraphLaunch(h->gexec, h->stream));
+    h->launches += 0;  // counted below from the iteration count
+  } else {
+    launch(h, K_PREPARE, -1, [&] { launch_prepare(p, h->stream); });
     CK(cudaGetLastError());
-    launched += batch;
-    CK(cudaMemcpyAsync(h->h_st, h->st.p, sizeof(DevState), cudaMemcpyDeviceToHost,
-                       h->stream));
-    CK(cudaStreamSynchronize(h->stream));
-    if (h->h_st->done) break;
-    if (launched >= h->max_iter) break;
-    batch = 2;
+    // Kernels exit immediately once the device sets `done`, so iterations
+    // are enqueued speculatively in batches and the flag is read once per
+    // batch (the minimum run length is itrPat + 1).
+    int launched = 0;
+    int batch = itrPat + 1;
+    for (;;) {
+      for (int b = 0; b < batch; ++b) {
+        const int iter = launched + b;
+        launch(h, K_LOC, iter, [&] { launch_locality(p, ps, h->stream); });
+        if (!p.fuse_tail) TRY(split_tail(h, p, TAIL_LOC, iter));
+        launch(h, K_ASG, iter, [&] { launch_assign(p, ps, h->stream); });
+        if (!p.fuse_tail) TRY(split_tail(h, p, TAIL_ASG, iter));
+        launch(h, K_COST, iter, [&] { launch_cost(p, ps, h->stream); });
+        if (!p.fuse_tail) TRY(split_tail(h, p, TAIL_COST, iter));
+      }
+      CK(cudaGetLastError());
+      launched += batch;
+      CK(cudaMemcpyAsync(h->h_st, h->st.p, sizeof(DevState), cudaMemcpyDeviceToHost,
+                         h->stream));
+      CK(cudaStreamSynchronize(h->stream));
+      if (h->h_st->done) break;
+      if (launched >= h->max_iter) break;
+      batch = 2;
+    }
+    // Refinement phase (Alg 1 l.16-19)
+    launch(h, K_REF, -1, [&] { launch_refine_x(p, ps, h->stream); });
+    if (!p.fuse_tail) TRY(split_tail(h, p, TAIL_REF, -1));
+    launch(h, K_FIN, -1, [&] { launch_final(p, ps, h->stream); });
+    CK(cudaGetLastError());
   }
-  // Refinement phase (Alg 1 l.16-19)
-  launch(h, K_REF, -1, [&] { launch_refine_x(p, ps, h->stream); });
-  if (!p.fuse_tail) TRY(split_tail(h, p, ps, TAIL_REF, -1));
-  launch(h, K_FIN, -1, [&] { launch_final(p, ps, h->stream); });
-  CK(cudaGetLastError());
   CK(cudaMemcpyAsync(h->h_st, h->st.p, sizeof(DevState), cudaMemcpyDeviceToHost, h->stream));
   if (out) {
     if (out->labels && !out->labels_on_device)
@@ -633,19 +751,21 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
                          h->stream));
   }
   CK(cudaStreamSynchronize(h->stream));
+  if (h->h_st->err) return fail(PROCLUS_EINTERNAL, "device reported error %d", h->h_st->err);
+  const int T = h->h_st->iterations;
+  if (use_graph) h->launches += 1 + 3 * (int64_t)T + 2;
   if (out) {
     for (int i = 0; i < k; ++i)
       if (out->medoids) out->medoids[i] = h->h_mids[(size_t)h->h_st->mbest[i]];
     out->cost = h->h_st->cost_best;
-    out->iterations = h->h_st->iterations;
+    out->iterations = T;
   }
   h->last_k = k;
-  h->tr_count = h->trace ? std::min(h->h_st->iterations, h->tr_cap) : 0;
+  h->tr_count = h->trace ? std::min(T, h->tr_cap) : 0;
   if (h->stats) {
     proclus_stats& S = h->last_stats;
-    const int T = h->h_st->iterations;
     const double bytes_pass = 4.0 * (double)h->n * d + (double)h->n;  // data + u8 labels
-    float first = 0.f;
+    float last = 0.f;
     for (size_t r = h->rec_done; r < h->recs.size(); ++r) {
       const auto& R = h->recs[r];
       if (R.iter >= T) continue;  // speculative launch after the stop: no work
@@ -655,16 +775,20 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
       S.ms[R.kind] += ms;
       float from0 = 0.f;
       CK(cudaEventElapsedTime(&from0, h->recs[0].a, R.b));
-      if (from0 > first) first = from0;
+      if (from0 > last) last = from0;
     }
     h->rec_done = h->recs.size();
-    if (first > S.run_ms) S.run_ms = first;
+    if (last > S.run_ms) S.run_ms = last;
     S.alg_bytes[K_LOC] += h->h_st->bytes_loc;
     S.alg_bytes[K_ASG] += T * bytes_pass;
     S.alg_bytes[K_COST] += T * bytes_pass;
     S.alg_bytes[K_REF] += bytes_pass;
     S.alg_bytes[K_FIN] += 4.0 * (double)h->n * d + 4.0 * (double)h->n;
     S.total_launches = h->launches;
+    for (int t = 0; t < 4; ++t) {
+      S.tail_ms[t] += (double)h->h_st->tail_ns[t] * 1e-6;
+      S.fallbacks[t] += h->h_st->fallback[t];
+    }
   }
   return PROCLUS_OK;
 }
@@ -672,8 +796,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
 extern "C" {
 
 proclus_status proclus_run(proclus_handle* h, int32_t k, int32_t l, int32_t A, int32_t B,
-                           double minDev, int32_t itrPat, uint64_t seed,
-                           proclus_result* out) {
+                           double minDev, int32_t itrPat, uint64_t seed, proclus_result* out) {
   if (!h) return fail(PROCLUS_EINVAL, "handle is NULL");
   if (!out || !out->medoids || !out->dims || !out->labels)
     return fail(PROCLUS_EINVAL, "out and its labels/medoids/dims arrays are required");

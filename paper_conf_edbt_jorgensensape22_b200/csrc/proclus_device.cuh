@@ -9,18 +9,22 @@
 namespace pc {
 
 constexpr int KMAX = 32;    // k <= 32: per-point medoid membership is a u32
-constexpr int WMAX = 8;     // warps per pass block (P <= 256)
-constexpr int PMAX = 256;   // points per streamed chunk
+constexpr int TPB_MAX = 512;
+constexpr int WMAX = 8;     // warps per pass block
+constexpr int UMAX = 4;     // points per thread in a chunk
+constexpr int SMAX = 3;     // max bulk-copy ring depth
+constexpr int NCOPY = 8;    // copies of the global accumulators (atomic spread)
+constexpr int DREG = 32;    // d <= DREG: a point's coordinates live in registers
+constexpr int PAD_ALIGN = 1024;  // n_pad multiple; shard boundaries for invariance
 
 // One medoid slot whose locality set changes in this iteration
 // (GPU-FAST-PROCLUS).  The band is (lo, hi]: Theorem 3.1 / eq 3.
 struct ActSlot {
   int slot;      // cluster slot i in MCur
   int mpos;      // MIdx_i: position in M, row of Dist and H
-  int compute;   // 1: DistFound is false -> compute and store Dist row
+  int compute;   // 1: DistFound is false -> compute and store the Dist row
   int lam;       // lambda_i (eq 6): +1 grow, -1 shrink
   double lo, hi; // band (lo, hi]; lo = -inf on first use (L_i itself)
-  float lo32, hi32;  // round-to-nearest fp32 of lo / hi (cached-row test)
 };
 
 // Mutable control state of one run, resident in device memory so that the
@@ -40,6 +44,8 @@ struct DevState {
   unsigned int ticket[4];       // last-block tickets of the pass kernels
   int err;
   double bytes_loc;             // algorithmic bytes of the locality passes
+  long long fallback[4];        // exact fp64 re-decisions (loc, asg, fin, -)
+  unsigned long long tail_ns[4];  // %globaltimer time in the single-block tails
 };
 
 struct TraceBufs {
@@ -57,16 +63,16 @@ struct TraceBufs {
 
 struct RunParams {
   long long n;        // rows on this device
-  long long n_pad;    // padded row count of the SoA layout (multiple of PMAX)
+  long long n_pad;    // padded row count of the SoA layout (multiple of PAD_ALIGN)
   long long n_total;  // |Data| (all ranks): threshold of P:91 and eq 8
   int d, k, l, nM, itrPat, max_iter, metric;
   double minDev;
   const float* xs;         // data, SoA [d][n_pad] fp32
   const float* mrows;      // rows of M [nM][d] fp32
-  float* dist;             // Dist cache [nM][n_pad] fp32
+  float* dist;             // Dist cache [nM][n_pad] fp32, certified values
   unsigned char* lab0;     // label buffers (current / best, swapped by index)
   unsigned char* lab1;
-  double* H;               // [nM][d] (eq 5)
+  long long* Hq;           // [nM][d] H of eq 5 in fixed point (scale 2^e_j)
   double* dprev;           // [nM] delta' of the previous use
   long long* nL;           // [nM] |L|
   unsigned char* found;    // [nM] DistFound
@@ -77,15 +83,18 @@ struct RunParams {
   double* X;               // [k][d]
   double* Z;               // [k][d] scratch
   double* mu;              // [k][d] centroid on D_i, index (i, t)
-  double* part;            // [grid][k*d] per-block partial sums
-  long long* partc;        // [grid][KMAX] per-block partial counts
-  double* red;             // [k*d] reduced sums (after allreduce)
-  long long* redc;         // [KMAX]
+  long long* accg;         // [NCOPY][k*d] global fixed-point cell sums (atomics)
+  long long* cntg;         // [NCOPY][KMAX] global counts
+  const double* scale;     // [d] 2^e_j   (fixed-point scale of dimension j)
+  const double* iscale;    // [d] 2^-e_j
   int* pool;               // [nM] scratch of the replacement step
   DevState* st;
-  int P;                   // points per chunk == blockDim.x of pass kernels
+  int P;                   // points per chunk (threads per block = P / PPT)
+  int stages;              // ring depth (2 or 3)
   long long nchunks;
   int fuse_tail;           // 1: last block finalises (single GPU)
+  int use_cond;            // 1: running inside a graph while-node
+  unsigned long long cond; // cudaGraphConditionalHandle
   TraceBufs tr;
   int* out_labels;         // final labels [n] int32 (refinement)
   double* Delta;           // [k] outlier radii
@@ -101,16 +110,16 @@ __device__ __forceinline__ double ddiv(double a, double b) { return __ddiv_rn(a,
 
 // Full-space distance ||p - q||: L2 = sqrt(sum_j (p_j - q_j)^2), L1
 // = sum_j |p_j - q_j|, j ascending.  p has stride ps, q stride 1.
-__device__ __forceinline__ double full_dist(const double* p, int ps,
-                                            const double* q, int d,
+template <class TP, class TQ>
+__device__ __forceinline__ double full_dist(const TP* p, int ps, const TQ* q, int d,
                                             int metric) {
   double s = 0.0;
   if (metric == 1) {
-    for (int j = 0; j < d; ++j) s = dadd(s, fabs(dsub(p[j * ps], q[j])));
+    for (int j = 0; j < d; ++j) s = dadd(s, fabs(dsub((double)p[j * ps], (double)q[j])));
     return s;
   }
   for (int j = 0; j < d; ++j) {
-    double t = dsub(p[j * ps], q[j]);
+    double t = dsub((double)p[j * ps], (double)q[j]);
     s = dadd(s, dmul(t, t));
   }
   return __dsqrt_rn(s);

@@ -1,44 +1,100 @@
 // proclus_kernels.cu -- sm_100a kernels of the PROCLUS hot path
 // (GPU-FAST-PROCLUS, section 4, re-designed for B200).
 //
-// Every per-iteration pass is a persistent, chunk-streaming kernel: the grid
-// is a multiple of the SM count, block b owns the chunks b, b+G, b+2G, ...
-// of P consecutive points (a static schedule, so every partial sum has a
-// fixed reduction order and the whole run is deterministic).  A chunk is
-// staged in shared memory as fp64 (one coalesced fp32 load per dimension and
-// point, SoA layout), the per-point decisions are taken by one thread per
-// point in exactly the oracle's fp64 arithmetic, and the per-(cluster,
-// dimension) sums are computed by "cells": one thread per (i, j) walks the
-// compacted member list of cluster / band i inside the chunk.  No floating
-// point atomics anywhere.  The last block to finish reduces the per-block
-// partials in block order and runs the small single-block step of the
-// algorithm that follows (finalise H and select dimensions, centroids, cost
-// and the Alg 1 l.10-14 control), so an iteration is three launches.
+// Every per-iteration pass is a persistent kernel that streams the data in
+// chunks of P points (SoA fp32, one 1-D bulk copy per dimension row) through
+// a 2-3 stage shared-memory ring filled by cp.async.bulk (TMA) and tracked by
+// mbarriers, so HBM traffic overlaps the compute of the previous chunks.
+// Chunks are small (P = 128 points for d <= 64) so that 4-8 blocks share an
+// SM and one block's barriers are hidden by the others.  Block b owns chunks
+// b, b+G, ...; inside a chunk
+//  (A) one thread per point takes the per-point decision (ComputeL band
+//      membership, AssignPoints argmin) in fp32 with a certified error bound
+//      and falls back to the oracle's exact fp64 expression only when the
+//      fp32 value is within that bound of the threshold / runner-up;
+//  (B) the per-point decisions are compacted into per-set member lists;
+//  (C) "cells" (S threads per (set, dimension)) sum over their list in fp64
+//      and quantise the chunk's sum to int64 fixed point (scale 2^e_j per
+//      dimension), accumulated exactly in shared memory and finally with one
+//      int64 atomicAdd per cell per block into one of NCOPY global copies.
+//      Integer addition is associative, so the totals do not depend on block
+//      scheduling, grid size or the number of GPUs: runs are bit-reproducible.
+// The last block to finish (ticket) runs the small single-block step that
+// follows (finalise H and select dimensions / centroids / cost and the
+// Alg 1 l.10-14 control), so an iteration is three launches; inside a CUDA
+// graph while-node the cost tail also sets the loop condition.
 #include <math_constants.h>
 
 #include "proclus_kernels.h"
 
 namespace pc {
 
+// ===================================================================== PTX
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+  return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phase) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes,
+                                         unsigned long long* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
 // ===================================================================== N0
+// row-major [n][d] -> SoA [d][n_pad] (zero padding), non-finite flag and the
+// per-dimension max |x| (as float bits; non-negative floats order as uints).
 __global__ void k_pack_soa(const float* __restrict__ in, long long n, int d,
-                           long long n_pad, float* __restrict__ xs, int* bad) {
+                           long long n_pad, float* __restrict__ xs, int* bad,
+                           unsigned* colmax) {
   __shared__ float tile[32][33];
   const long long p0 = (long long)blockIdx.x * 32;
   const int j0 = blockIdx.y * 32;
   const int tx = threadIdx.x, ty = threadIdx.y;
   int nonfinite = 0;
+  float amax = 0.f;
   for (int r = ty; r < 32; r += 8) {
     long long p = p0 + r;
     int j = j0 + tx;
     float v = 0.f;
     if (p < n && j < d) {
       v = in[p * d + j];
-      if (!isfinite(v)) nonfinite = 1;
+      if (!isfinite(v))
+        nonfinite = 1;
+      else
+        amax = fmaxf(amax, fabsf(v));
     }
     tile[r][tx] = v;
   }
   if (nonfinite) atomicOr(bad, 1);
+  if (j0 + tx < d && amax > 0.f) atomicMax(colmax + j0 + tx, __float_as_uint(amax));
   __syncthreads();
   for (int r = ty; r < 32; r += 8) {
     int j = j0 + r;
@@ -47,16 +103,15 @@ __global__ void k_pack_soa(const float* __restrict__ in, long long n, int d,
   }
 }
 
-void launch_pack_soa(const float* in, long long n, int d, long long n_pad,
-                     float* xs, int* bad, cudaStream_t s) {
+void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
+                     unsigned* colmax, cudaStream_t s) {
   dim3 grid((unsigned)((n_pad + 31) / 32), (unsigned)((d + 31) / 32));
-  k_pack_soa<<<grid, dim3(32, 8), 0, s>>>(in, n, d, n_pad, xs, bad);
+  k_pack_soa<<<grid, dim3(32, 8), 0, s>>>(in, n, d, n_pad, xs, bad, colmax);
 }
 
-__global__ void k_gather_rows(const float* __restrict__ xs, long long n_pad,
-                              int d, const long long* __restrict__ ids,
-                              long long row_offset, long long n_local, int cnt,
-                              float* __restrict__ out) {
+__global__ void k_gather_rows(const float* __restrict__ xs, long long n_pad, int d,
+                              const long long* __restrict__ ids, long long row_offset,
+                              long long n_local, int cnt, float* __restrict__ out) {
   const long long tot = (long long)cnt * d;
   for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < tot;
        e += (long long)gridDim.x * blockDim.x) {
@@ -66,19 +121,17 @@ __global__ void k_gather_rows(const float* __restrict__ xs, long long n_pad,
   }
 }
 
-void launch_gather_rows(const float* xs, long long n_pad, int d,
-                        const long long* ids, long long row_offset,
-                        long long n_local, int cnt, float* out, cudaStream_t s) {
+void launch_gather_rows(const float* xs, long long n_pad, int d, const long long* ids,
+                        long long row_offset, long long n_local, int cnt, float* out,
+                        cudaStream_t s) {
   long long tot = (long long)cnt * d;
   int blocks = (int)((tot + 255) / 256);
   if (blocks < 1) blocks = 1;
   if (blocks > 1184) blocks = 1184;
-  k_gather_rows<<<blocks, 256, 0, s>>>(xs, n_pad, d, ids, row_offset, n_local,
-                                       cnt, out);
+  k_gather_rows<<<blocks, 256, 0, s>>>(xs, n_pad, d, ids, row_offset, n_local, cnt, out);
 }
 
-__global__ void k_gather_m(const float* __restrict__ srows,
-                           const long long* __restrict__ sids,
+__global__ void k_gather_m(const float* __restrict__ srows, const long long* __restrict__ sids,
                            const int* __restrict__ spos, int nM, int d,
                            float* __restrict__ mrows, long long* __restrict__ mids) {
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < nM * d;
@@ -89,9 +142,8 @@ __global__ void k_gather_m(const float* __restrict__ srows,
   }
 }
 
-void launch_gather_m(const float* srows, const long long* sids, const int* spos,
-                     int nM, int d, float* mrows, long long* mids,
-                     cudaStream_t s) {
+void launch_gather_m(const float* srows, const long long* sids, const int* spos, int nM, int d,
+                     float* mrows, long long* mids, cudaStream_t s) {
   int blocks = (nM * d + 255) / 256;
   if (blocks < 1) blocks = 1;
   if (blocks > 592) blocks = 592;
@@ -99,211 +151,260 @@ void launch_gather_m(const float* srows, const long long* sids, const int* spos,
 }
 
 // ===================================================================== N1
-// Greedy (Alg 2) in a single CTA: all #M-1 dependent picks in one
-// launch instead of two launches per pick.  dist[q] is the min distance of
-// S-position q to the picked set (-1 once picked, reading R7); the argmax
-// prefers the larger value, then the smaller position.
-__device__ __forceinline__ void argmax_merge(double& v, int& q, double v2, int q2) {
-  if (v2 > v || (v2 == v && q2 < q)) {
-    v = v2;
-    q = q2;
+// Greedy (Alg 2).  Step 1 (whole GPU): the exact fp64 distance
+// matrix Ds[a][q] = full(S_q, S_a) of the sample, in the oracle's expression
+// (all #M picks read rows of it).  Step 2 (one CTA, all #M-1 dependent picks
+// in one launch; the paper uses two launches per pick): dist[q] =
+// min(dist[q], Ds[pick][q]) and a block argmax (larger distance, then smaller
+// position, reading R7) with redux.sync on a 64-bit order key: 0 for picked
+// points, bits(dist) + 1 otherwise.
+constexpr int GR_TPB = 1024;
+constexpr int GR_PPT = 4;   // S-positions per thread in registers (nS <= 4096)
+
+__global__ void k_sdist(const float* __restrict__ srows, int nS, int d, int metric,
+                        double* __restrict__ Ds) {
+  const long long tot = (long long)nS * nS;
+  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < tot;
+       e += (long long)gridDim.x * blockDim.x) {
+    const int a = (int)(e / nS), q = (int)(e - (long long)a * nS);
+    Ds[e] = full_dist(srows + (long long)q * d, 1, srows + (long long)a * d, d, metric);
   }
 }
 
-__global__ void __launch_bounds__(1024)
-    k_greedy(const float* __restrict__ srows, int nS, int d, int nM, int q0,
-             int metric, int rows_in_smem, int* __restrict__ spos,
+struct KeyIdx {
+  unsigned hi, lo, idx;
+};
+
+__device__ __forceinline__ KeyIdx warp_argmax(unsigned hi, unsigned lo, unsigned idx) {
+  const unsigned full = 0xffffffffu;
+  unsigned mhi = __reduce_max_sync(full, hi);
+  unsigned mlo = __reduce_max_sync(full, hi == mhi ? lo : 0u);
+  unsigned midx = __reduce_min_sync(full, (hi == mhi && lo == mlo) ? idx : 0xffffffffu);
+  return {mhi, mlo, midx};
+}
+
+__device__ __forceinline__ unsigned long long dkey(double v) {
+  return v >= 0.0 ? (unsigned long long)__double_as_longlong(v) + 1ull : 0ull;
+}
+
+// 256 threads x 16 positions in registers; one barrier per pick: every warp
+// publishes its candidate in a parity-double-buffered slot and then all
+// warps reduce the 8 candidates redundantly.
+constexpr int GM_TPB = 256;
+constexpr int GM_PPT = 16;
+__global__ void __launch_bounds__(GM_TPB)
+    k_greedy(const double* __restrict__ Ds, int nS, int nM, int q0, int* __restrict__ spos,
              double* __restrict__ pickdist) {
-  extern __shared__ double gsm[];
-  double* dist = gsm;                               // [nS]
-  double* prow = gsm + nS;                          // [d] picked row
-  double* rows = prow + d;                          // [nS][d] if cached
-  __shared__ double wv[32];
-  __shared__ int wq[32];
-  __shared__ int pick;
-  const int tid = threadIdx.x, bd = blockDim.x;
-  const int lane = tid & 31, w = tid >> 5, nw = (bd + 31) >> 5;
-
-  if (rows_in_smem)
-    for (int e = tid; e < nS * d; e += bd) rows[e] = (double)srows[e];
-  for (int j = tid; j < d; j += bd) prow[j] = (double)srows[(long long)q0 * d + j];
-  __syncthreads();
-
-  auto dist_to_pick = [&](int q) -> double {
-    if (rows_in_smem) return full_dist(rows + (long long)q * d, 1, prow, d, metric);
-    const float* r = srows + (long long)q * d;
-    double s = 0.0;
-    if (metric == 1) {
-      for (int j = 0; j < d; ++j) s = dadd(s, fabs(dsub((double)r[j], prow[j])));
-      return s;
-    }
-    for (int j = 0; j < d; ++j) {
-      double t = dsub((double)r[j], prow[j]);
-      s = dadd(s, dmul(t, t));
-    }
-    return __dsqrt_rn(s);
-  };
-
-  for (int q = tid; q < nS; q += bd) dist[q] = (q == q0) ? -1.0 : dist_to_pick(q);
+  __shared__ unsigned whi[2][8], wlo[2][8], widx[2][8];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  constexpr int nw = GM_TPB / 32;
+  double dreg[GM_PPT];
+#pragma unroll
+  for (int t = 0; t < GM_PPT; ++t) {
+    const int q = tid + t * GM_TPB;
+    dreg[t] = (q < nS && q != q0) ? __ldg(Ds + (long long)q0 * nS + q) : -1.0;
+  }
   if (tid == 0) {
     spos[0] = q0;
     if (pickdist) pickdist[0] = CUDART_INF;
   }
   for (int i = 1; i < nM; ++i) {
-    __syncthreads();
-    double v = -2.0;
-    int q = 0x7fffffff;
-    for (int t = tid; t < nS; t += bd) argmax_merge(v, q, dist[t], t);
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      double v2 = __shfl_down_sync(0xffffffffu, v, o);
-      int q2 = __shfl_down_sync(0xffffffffu, q, o);
-      argmax_merge(v, q, v2, q2);
+    for (int t = 0; t < GM_PPT; ++t) {
+      const unsigned long long key = dkey(dreg[t]);
+      if (key > bk) {  // ascending q: strict > keeps the smaller position
+        bk = key;
+        bq = tid + t * GM_TPB;
+      }
     }
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    const int par = i & 1;
     if (lane == 0) {
-      wv[w] = v;
-      wq[w] = q;
+      whi[par][w] = r.hi;
+      wlo[par][w] = r.lo;
+      widx[par][w] = r.idx;
+    }
+    __syncthreads();
+    KeyIdx s = warp_argmax(lane < nw ? whi[par][lane] : 0u, lane < nw ? wlo[par][lane] : 0u,
+                           lane < nw ? widx[par][lane] : 0xffffffffu);
+    const int qs = (int)s.idx;
+    if (tid == 0) {
+      spos[i] = qs;
+      if (pickdist) {
+        unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
+        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+      }
+    }
+    const double* row = Ds + (long long)qs * nS;
+#pragma unroll
+    for (int t = 0; t < GM_PPT; ++t) {
+      const int q = tid + t * GM_TPB;
+      if (q == qs) {
+        dreg[t] = -1.0;
+      } else if (dreg[t] >= 0.0) {
+        const double u = __ldg(row + q);
+        if (u < dreg[t]) dreg[t] = u;
+      }
+    }
+  }
+}
+
+// Large samples (#S > 4096): same picks, distances computed on the fly.
+__global__ void __launch_bounds__(GR_TPB)
+    k_greedy_big(const float* __restrict__ srows, int nS, int d, int nM, int q0, int metric,
+                 double* __restrict__ dist, int* __restrict__ spos, double* __restrict__ pickdist) {
+  extern __shared__ double prow[];
+  __shared__ unsigned whi[32], wlo[32], widx[32];
+  __shared__ int pick_s;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const int nw = GR_TPB / 32;
+  for (int j = tid; j < d; j += GR_TPB) prow[j] = (double)srows[(long long)q0 * d + j];
+  __syncthreads();
+  for (int q = tid; q < nS; q += GR_TPB)
+    dist[q] = (q == q0) ? -1.0 : full_dist(srows + (long long)q * d, 1, prow, d, metric);
+  if (tid == 0) {
+    spos[0] = q0;
+    if (pickdist) pickdist[0] = CUDART_INF;
+  }
+  for (int i = 1; i < nM; ++i) {
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
+    for (int q = tid; q < nS; q += GR_TPB) {
+      const unsigned long long key = dkey(dist[q]);
+      if (key > bk) {
+        bk = key;
+        bq = q;
+      }
+    }
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    if (lane == 0) {
+      whi[w] = r.hi;
+      wlo[w] = r.lo;
+      widx[w] = r.idx;
     }
     __syncthreads();
     if (w == 0) {
-      v = lane < nw ? wv[lane] : -2.0;
-      q = lane < nw ? wq[lane] : 0x7fffffff;
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        double v2 = __shfl_down_sync(0xffffffffu, v, o);
-        int q2 = __shfl_down_sync(0xffffffffu, q, o);
-        argmax_merge(v, q, v2, q2);
-      }
+      KeyIdx s = warp_argmax(lane < nw ? whi[lane] : 0u, lane < nw ? wlo[lane] : 0u,
+                             lane < nw ? widx[lane] : 0xffffffffu);
       if (lane == 0) {
-        pick = q;
-        spos[i] = q;
-        if (pickdist) pickdist[i] = v;
+        pick_s = (int)s.idx;
+        spos[i] = (int)s.idx;
+        if (pickdist) {
+          unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
+          pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+        }
       }
     }
     __syncthreads();
-    const int qs = pick;
-    for (int j = tid; j < d; j += bd)
-      prow[j] = rows_in_smem ? rows[(long long)qs * d + j]
-                             : (double)srows[(long long)qs * d + j];
+    const int qs = pick_s;
+    for (int j = tid; j < d; j += GR_TPB) prow[j] = (double)srows[(long long)qs * d + j];
     __syncthreads();
-    for (int t = tid; t < nS; t += bd) {
-      if (t == qs) {
-        dist[t] = -1.0;
-      } else if (dist[t] >= 0.0) {
-        double u = dist_to_pick(t);
-        if (u < dist[t]) dist[t] = u;
+    for (int q = tid; q < nS; q += GR_TPB) {
+      if (q == qs) {
+        dist[q] = -1.0;
+      } else if (dist[q] >= 0.0) {
+        const double u = full_dist(srows + (long long)q * d, 1, prow, d, metric);
+        if (u < dist[q]) dist[q] = u;
       }
     }
+    __syncthreads();
   }
 }
 
-cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0,
-                          int metric, int* spos, double* pickdist,
-                          cudaStream_t s) {
-  size_t base = sizeof(double) * ((size_t)nS + d);
-  size_t rows = sizeof(double) * (size_t)nS * d;
-  int in_smem = base + rows <= 200 * 1024;
-  size_t smem = base + (in_smem ? rows : 0);
-  cudaError_t e = cudaFuncSetAttribute(k_greedy,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)smem);
-  if (e != cudaSuccess) return e;
-  k_greedy<<<1, 1024, smem, s>>>(srows, nS, d, nM, q0, metric, in_smem, spos,
-                                 pickdist);
+size_t greedy_scratch_doubles(int nS) {
+  return nS <= GM_PPT * GM_TPB ? (size_t)nS * nS : (size_t)nS;
+}
+
+cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
+                          double* scratch, int* spos, double* pickdist, cudaStream_t s) {
+  if (nS <= GM_PPT * GM_TPB) {
+    const long long tot = (long long)nS * nS;
+    int blocks = (int)((tot + 255) / 256);
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    if (blocks < 1) blocks = 1;
+    k_sdist<<<blocks, 256, 0, s>>>(srows, nS, d, metric, scratch);
+    k_greedy<<<1, GM_TPB, 0, s>>>(scratch, nS, nM, q0, spos, pickdist);
+  } else {
+    k_greedy_big<<<1, GR_TPB, sizeof(double) * d, s>>>(srows, nS, d, nM, q0, metric, scratch,
+                                                       spos, pickdist);
+  }
   return cudaGetLastError();
 }
 
-// ============================================================ block helpers
-// Shared scratch for compacting per-point membership bitmasks into per-set
-// member lists (ascending point order inside the chunk).
-struct ListScratch {
-  unsigned* ballot;   // [KMAX][WMAX]
-  int* woff;          // [KMAX][WMAX]
-  int* cnt;           // [KMAX]
-  int* base;          // [KMAX]
-  unsigned short* list;  // [sum of counts]
+// ============================================================ pipeline
+// Warp-specialised chunk pipeline: the last warp of a block is the TMA
+// producer, the other NW warps consume.  full[s] completes when the bulk
+// copies of a chunk landed (expect_tx); empty[s] completes when all NW
+// consumer warps released the stage (one arrive each), after which the
+// producer refills it.  No block-wide barrier inside the chunk loop.
+__device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+struct ExtraRows {
+  int n;
+  const float* src[KMAX];  // global row bases (indexed by point)
 };
 
-__device__ void build_lists(unsigned mask, int nsets, ListScratch ls) {
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int W = blockDim.x >> 5;
-  for (int a = 0; a < nsets; ++a) {
-    unsigned b = __ballot_sync(0xffffffffu, (mask >> a) & 1u);
-    if (lane == 0) ls.ballot[a * WMAX + w] = b;
-  }
-  __syncthreads();
-  if (threadIdx.x < nsets) {
-    const int a = threadIdx.x;
-    int tot = 0;
-    for (int v = 0; v < W; ++v) {
-      ls.woff[a * WMAX + v] = tot;
-      tot += __popc(ls.ballot[a * WMAX + v]);
-    }
-    ls.cnt[a] = tot;
-  }
-  __syncthreads();
+struct Pipe {
+  float* buf;                 // [stages][rows][P]
+  unsigned char* lab;         // [stages][P] (label passes) or nullptr
+  unsigned long long* full;   // [SMAX]
+  unsigned long long* empty;  // [SMAX]
+  int rows;
+};
+
+__device__ __forceinline__ void pipe_init(const RunParams& p, const Pipe& R, int nw) {
   if (threadIdx.x == 0) {
-    int s = 0;
-    for (int a = 0; a < nsets; ++a) {
-      ls.base[a] = s;
-      s += ls.cnt[a];
+    for (int s = 0; s < p.stages; ++s) {
+      mbar_init(&R.full[s], 1);
+      mbar_init(&R.empty[s], (unsigned)nw);
     }
+    fence_mbar_init();
   }
-  __syncthreads();
-  const unsigned lt = (1u << lane) - 1u;
-  unsigned m = mask;
-  while (m) {
-    const int a = __ffs(m) - 1;
-    m &= m - 1u;
-    int pos = ls.base[a] + ls.woff[a * WMAX + w] +
-              __popc(ls.ballot[a * WMAX + w] & lt);
-    ls.list[pos] = (unsigned short)threadIdx.x;
-  }
-  __syncthreads();
 }
 
-// sum_{t < cnt} f(x[L[t]]) with four interleaved partial sums combined in a
-// fixed order (deterministic).  MODE 0: x, MODE 1: |x - c|.
-template <int MODE>
-__device__ __forceinline__ double list_sum(const double* __restrict__ xr,
-                                           const unsigned short* __restrict__ L,
-                                           int cnt, double c) {
-  double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
-  int t = 0;
-  for (; t + 4 <= cnt; t += 4) {
-    double v0 = xr[L[t]], v1 = xr[L[t + 1]], v2 = xr[L[t + 2]], v3 = xr[L[t + 3]];
-    if (MODE == 1) {
-      v0 = fabs(dsub(v0, c));
-      v1 = fabs(dsub(v1, c));
-      v2 = fabs(dsub(v2, c));
-      v3 = fabs(dsub(v3, c));
+// Producer warp: stream this block's chunks b, b+G, ... through the ring.
+__device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
+                             const unsigned char* labsrc, const ExtraRows* ex) {
+  const int lane = threadIdx.x & 31;
+  const unsigned row = (unsigned)p.P * 4u;
+  const int nex = ex ? ex->n : 0;
+  const unsigned bytes = row * (unsigned)(p.d + nex) + (labsrc ? (unsigned)p.P : 0u);
+  for (long long i = 0; i < nmy; ++i) {
+    const int stg = (int)(i % p.stages);
+    if (i >= p.stages) {  // the consumers of chunk i - stages released this stage
+      mbar_wait(&R.empty[stg], (unsigned)(((i / p.stages) - 1) & 1));
+      fence_proxy_async();
     }
-    s0 = dadd(s0, v0);
-    s1 = dadd(s1, v1);
-    s2 = dadd(s2, v2);
-    s3 = dadd(s3, v3);
+    const long long base = (blockIdx.x + i * gridDim.x) * (long long)p.P;
+    if (lane == 0) mbar_expect_tx(&R.full[stg], bytes);
+    __syncwarp();
+    float* dst = R.buf + (size_t)stg * R.rows * p.P;
+    for (int j = lane; j < p.d + nex; j += 32) {
+      const float* src = j < p.d ? p.xs + (size_t)j * p.n_pad + base : ex->src[j - p.d] + base;
+      bulk_g2s(dst + (size_t)j * p.P, src, row, &R.full[stg]);
+    }
+    if (labsrc && lane == 0)
+      bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, &R.full[stg]);
   }
-  for (; t < cnt; ++t) {
-    double v = xr[L[t]];
-    if (MODE == 1) v = fabs(dsub(v, c));
-    s0 = dadd(s0, v);
-  }
-  return dadd(dadd(s0, s1), dadd(s2, s3));
 }
 
-// Stage one chunk (P points, all d dimensions) as fp64: x_s[j*(P+1) + p].
-__device__ __forceinline__ void stage_chunk(const float* __restrict__ xs,
-                                            long long n_pad, int d,
-                                            long long base, int P,
-                                            double* __restrict__ x_s) {
-  const int p = threadIdx.x;
-  const float* src = xs + base + p;
-#pragma unroll 4
-  for (int j = 0; j < d; ++j) x_s[j * (P + 1) + p] = (double)__ldg(src + (long long)j * n_pad);
+__device__ __forceinline__ void pipe_release(const Pipe& R, int stg) {
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) mbar_arrive(&R.empty[stg]);
 }
 
 // The last block to arrive (ticket) returns true; it then sees every other
-// block's partials (threadfence before the ticket, reads with ld.cg).
+// block's atomics (threadfence before the ticket, ld.cg reads after).
 __device__ bool last_block(unsigned int* ticket) {
   __shared__ int is_last;
   __threadfence();
@@ -320,21 +421,131 @@ __device__ bool last_block(unsigned int* ticket) {
   return is_last;
 }
 
-// Sum the per-block partials in block order into red / redc.
-__device__ void reduce_partials(const double* part, const long long* partc,
-                                int G, int stride, int ncell, int ncnt,
-                                double* red, long long* redc) {
+// Combine the per-warp accumulators (exact int64) and add them to one of the
+// NCOPY global copies with one atomic per non-zero cell.  Whole block.
+__device__ void flush_warps(const RunParams& p, const long long* acc_s, int nw, int ncap,
+                            int ncell, const long long* cnt_s, int ncnt) {
+  const int cp = blockIdx.x % NCOPY;
+  long long* acc = p.accg + (size_t)cp * p.k * p.d;
+  long long* cnt = p.cntg + (size_t)cp * KMAX;
   for (int c = threadIdx.x; c < ncell; c += blockDim.x) {
-    double s = 0.0;
-    for (int b = 0; b < G; ++b) s = dadd(s, __ldcg(part + (long long)b * stride + c));
-    red[c] = s;
+    long long s = 0;
+    for (int w = 0; w < nw; ++w) s += acc_s[w * ncap + c];
+    if (s) atomicAdd((unsigned long long*)&acc[c], (unsigned long long)s);
   }
   for (int c = threadIdx.x; c < ncnt; c += blockDim.x) {
     long long s = 0;
-    for (int b = 0; b < G; ++b) s += __ldcg(partc + (long long)b * KMAX + c);
-    redc[c] = s;
+    for (int w = 0; w < nw; ++w) s += cnt_s[w * KMAX + c];
+    if (s) atomicAdd((unsigned long long*)&cnt[c], (unsigned long long)s);
   }
-  __syncthreads();
+}
+
+// Exact total of accumulator c over the NCOPY copies; zeroes them.
+__device__ __forceinline__ long long take_acc(const RunParams& p, int c) {
+  long long s = 0;
+  const size_t stride = (size_t)p.k * p.d;
+  for (int q = 0; q < NCOPY; ++q) {
+    s += __ldcg(p.accg + q * stride + c);
+    p.accg[q * stride + c] = 0;
+  }
+  return s;
+}
+__device__ __forceinline__ long long take_cnt(const RunParams& p, int c) {
+  long long s = 0;
+  for (int q = 0; q < NCOPY; ++q) {
+    s += __ldcg(p.cntg + q * KMAX + c);
+    p.cntg[q * KMAX + c] = 0;
+  }
+  return s;
+}
+
+// One summation cell: set a (cluster / band slot), dimension j, centre c,
+// index of its accumulator.
+struct Cell {
+  int a, j, acc;
+  double c;
+};
+
+// Cells of one warp's sub-chunk (32*PPT points starting at q0): lane l owns
+// cells l, l+32, ...; the member set of a is the ballot bitmask bal[a*PPT+u]
+// of the warp's points.  fp64 sum (two interleaved accumulators, ascending
+// point order), quantised to int64 at scale 2^e_j and added to the lane's
+// own accumulator.  MODE 0: x, MODE 1: |x - c|.
+template <int MODE, int PPT>
+__device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, int q0,
+                                           const Cell* __restrict__ cells, int ncell,
+                                           const unsigned* __restrict__ bal,
+                                           long long* __restrict__ acc,
+                                           const double* __restrict__ scale_s) {
+  const int lane = threadIdx.x & 31;
+  for (int ci = lane; ci < ncell; ci += 32) {
+    const Cell C = cells[ci];
+    const float* xr = xs + (size_t)C.j * P + q0;
+    double s0 = 0.0, s1 = 0.0;
+#pragma unroll
+    for (int u = 0; u < PPT; ++u) {
+      unsigned m = bal[C.a * PPT + u];
+      const float* xu = xr + u * 32;
+      while (m) {
+        const int b0 = __ffs(m) - 1;
+        m &= m - 1u;
+        double v0 = (double)xu[b0];
+        if (MODE == 1) v0 = fabs(dsub(v0, C.c));
+        if (m) {
+          const int b1 = __ffs(m) - 1;
+          m &= m - 1u;
+          double v1 = (double)xu[b1];
+          if (MODE == 1) v1 = fabs(dsub(v1, C.c));
+          s1 = dadd(s1, v1);
+        }
+        s0 = dadd(s0, v0);
+      }
+    }
+    const double s = dadd(s0, s1);
+    if (s != 0.0) acc[C.acc] += __double2ll_rn(dmul(s, scale_s[C.j]));
+  }
+}
+
+// Publish one warp-uniform ballot per (set, u) for the cells of this warp.
+__device__ __forceinline__ void put_ballot(unsigned* bal, int idx, bool pred) {
+  const unsigned b = __ballot_sync(0xffffffffu, pred);
+  if ((threadIdx.x & 31) == 0) bal[idx] = b;
+}
+
+// ============================================================ smem carving
+struct Carve {
+  char* ptr;
+  __device__ explicit Carve(void* base) : ptr((char*)base) {}
+  template <class T>
+  __device__ T* take(size_t count) {
+    ptr = (char*)(((size_t)ptr + 15) & ~(size_t)15);
+    T* r = (T*)ptr;
+    ptr += sizeof(T) * count;
+    return r;
+  }
+};
+
+struct CarveSize {
+  size_t s = 0;
+  template <class T>
+  CarveSize& add(size_t count) {
+    s = ((s + 15) & ~(size_t)15) + sizeof(T) * count;
+    return *this;
+  }
+};
+
+__device__ Pipe carve_pipe(Carve& cv, const RunParams& p, int rows, bool with_lab) {
+  Pipe R;
+  R.rows = rows;
+  R.full = cv.take<unsigned long long>(SMAX);
+  R.empty = cv.take<unsigned long long>(SMAX);
+  R.buf = cv.take<float>((size_t)p.stages * rows * p.P);
+  R.lab = with_lab ? cv.take<unsigned char>((size_t)p.stages * p.P) : nullptr;
+  return R;
+}
+static void size_pipe(CarveSize& cs, int rows, int P, int stages, bool with_lab) {
+  cs.add<unsigned long long>(SMAX).add<unsigned long long>(SMAX).add<float>((size_t)stages * rows * P);
+  if (with_lab) cs.add<unsigned char>((size_t)stages * P);
 }
 
 // ============================================================ FindDimensions
@@ -349,7 +560,7 @@ __device__ void zscore_select(const double* X, int k, int d, int l, double* Z,
   __shared__ unsigned int hist[256];
   __shared__ unsigned long long prefix_s;
   __shared__ int need_s;
-  __shared__ int tcount[1024];
+  __shared__ int tcount[TPB_MAX];
   const int tid = threadIdx.x, bd = blockDim.x;
   const int kd = k * d;
   if (tid < k) {
@@ -386,7 +597,6 @@ __device__ void zscore_select(const double* X, int k, int d, int l, double* Z,
   __syncthreads();
   const int R = k * l - 2 * k;
   if (R > 0) {
-    // radix select of the R-th smallest key among the remaining cells
     if (tid == 0) {
       prefix_s = 0ull;
       need_s = R;
@@ -398,26 +608,43 @@ __device__ void zscore_select(const double* X, int k, int d, int l, double* Z,
       const unsigned long long pre = prefix_s;
       for (int c = tid; c < kd; c += bd) {
         if (dmask[c]) continue;
-        unsigned long long key = sortable_key(Z[c]);
+        const unsigned long long key = sortable_key(Z[c]);
         if ((key & hmask) == pre) atomicAdd(&hist[(key >> shift) & 255ull], 1u);
       }
       __syncthreads();
-      if (tid == 0) {
-        int need = need_s, cum = 0, b = 0;
-        for (b = 0; b < 256; ++b) {
-          if (cum + (int)hist[b] >= need) break;
-          cum += (int)hist[b];
+      if (tid < 32) {  // warp scan over 256 bins, 8 per lane
+        unsigned loc[8], tot = 0;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+          loc[b] = hist[tid * 8 + b];
+          tot += loc[b];
         }
-        need_s = need - cum;
-        prefix_s = pre | ((unsigned long long)b << shift);
+        unsigned x = tot;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          unsigned y = __shfl_up_sync(0xffffffffu, x, o);
+          if (tid >= o) x += y;
+        }
+        const unsigned before = x - tot;
+        const int need = need_s;
+        const bool here = (int)before < need && need <= (int)x;
+        const unsigned who = __ballot_sync(0xffffffffu, here);
+        if (here && tid == __ffs(who) - 1) {
+          unsigned cum = before;
+          int b = 0;
+          for (; b < 8; ++b) {
+            if ((int)(cum + loc[b]) >= need) break;
+            cum += loc[b];
+          }
+          need_s = need - (int)cum;
+          prefix_s = pre | ((unsigned long long)(tid * 8 + b) << shift);
+        }
       }
       hmask |= 255ull << shift;
       __syncthreads();
     }
     const unsigned long long K = prefix_s;
     const int need = need_s;  // how many cells with key == K to take
-    // cells with key < K are selected; of those equal to K the first `need`
-    // in (i, j) order.  Contiguous index ranges per thread + a scan.
     const int per = (kd + bd - 1) / bd;
     const int c0 = tid * per, c1 = min(kd, c0 + per);
     int eq = 0;
@@ -470,8 +697,7 @@ __device__ void prepare_iteration(const RunParams& p) {
     double m = CUDART_INF;
     for (int j = 0; j < k; ++j) {
       if (j == i) continue;
-      double t = full_dist(p.med + (long long)i * d, 1, p.med + (long long)j * d, d,
-                           p.metric);
+      double t = full_dist(p.med + (long long)i * d, 1, p.med + (long long)j * d, d, p.metric);
       if (t < m) m = t;
     }
     st->delta[i] = m;
@@ -497,14 +723,9 @@ __device__ void prepare_iteration(const RunParams& p) {
         a.lo = dl;
         a.hi = p.dprev[mp];
         a.lam = -1;
-      } else if (a.compute) {  // unreachable: used implies found
-        a.lo = -CUDART_INF;
-        a.hi = dl;
       } else {
         continue;  // delta unchanged: Delta L_i is empty (eq 3)
       }
-      a.lo32 = __double2float_rn(a.lo);
-      a.hi32 = __double2float_rn(a.hi);
       st->act[na++] = a;
     }
     st->n_act = na;
@@ -514,64 +735,28 @@ __device__ void prepare_iteration(const RunParams& p) {
 
 __global__ void k_prepare(RunParams p) { prepare_iteration(p); }
 
-void launch_prepare(const RunParams& p, cudaStream_t s) {
-  k_prepare<<<1, 256, 0, s>>>(p);
-}
-
-// ============================================================ smem carving
-struct Carve {
-  char* ptr;
-  __device__ explicit Carve(void* base) : ptr((char*)base) {}
-  template <class T>
-  __device__ T* take(size_t count) {
-    size_t a = alignof(T) < 8 ? 8 : alignof(T);
-    ptr = (char*)(((size_t)ptr + a - 1) & ~(a - 1));
-    T* r = (T*)ptr;
-    ptr += sizeof(T) * count;
-    return r;
-  }
-};
-
-static size_t carve_size(std::initializer_list<size_t> parts) {
-  size_t s = 0;
-  for (size_t b : parts) s += (b + 15) & ~(size_t)15;
-  return s + 64;
-}
-
-__device__ ListScratch carve_lists(Carve& cv, int list_len) {
-  ListScratch ls;
-  ls.ballot = cv.take<unsigned>(KMAX * WMAX);
-  ls.woff = cv.take<int>(KMAX * WMAX);
-  ls.cnt = cv.take<int>(KMAX);
-  ls.base = cv.take<int>(KMAX);
-  ls.list = cv.take<unsigned short>(list_len);
-  return ls;
-}
-
-static size_t lists_bytes(int list_len) {
-  return carve_size({sizeof(unsigned) * KMAX * WMAX, sizeof(int) * KMAX * WMAX,
-                     sizeof(int) * KMAX, sizeof(int) * KMAX,
-                     sizeof(unsigned short) * (size_t)list_len});
-}
+void launch_prepare(const RunParams& p, cudaStream_t s) { k_prepare<<<1, 256, 0, s>>>(p); }
 
 // ============================================================ tails
-// Locality tail: H and |L| updates of Theorem 3.2 / eq 6 and P:203, the
-// bookkeeping of DistFound / delta', X = H / |L|, FindDimensions.
+// Locality tail: H and |L| updates of Theorem 3.2 / eq 6 and P:203 (in fixed
+// point, so the incremental H is exact integer arithmetic), DistFound /
+// delta' bookkeeping, X = H / |L| and FindDimensions.
 __device__ void tail_locality(const RunParams& p) {
   DevState* st = p.st;
   const int d = p.d, na = st->n_act;
+  if (threadIdx.x == 0 && na > 0)  // byte model: data once + one Dist row per slot
+    st->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
   for (int c = threadIdx.x; c < na * d; c += blockDim.x) {
     const int a = c / d, j = c - a * d;
     const ActSlot A = st->act[a];
-    double* h = p.H + (long long)A.mpos * d + j;
-    *h = dadd(*h, A.lam > 0 ? p.red[c] : -p.red[c]);
+    const long long v = take_acc(p, c);
+    p.Hq[(long long)A.mpos * d + j] += (A.lam > 0 ? v : -v);
   }
   __syncthreads();
-  if (threadIdx.x == 0 && na > 0)  // byte model: data once + one Dist row per slot
-    st->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
   if (threadIdx.x < na) {
     const ActSlot A = st->act[threadIdx.x];
-    p.nL[A.mpos] += (A.lam > 0 ? p.redc[threadIdx.x] : -p.redc[threadIdx.x]);
+    const long long v = take_cnt(p, threadIdx.x);
+    p.nL[A.mpos] += (A.lam > 0 ? v : -v);
     p.dprev[A.mpos] = st->delta[A.slot];
     p.used[A.mpos] = 1;
     p.found[A.mpos] = 1;
@@ -581,12 +766,11 @@ __device__ void tail_locality(const RunParams& p) {
   for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
     const int i = c / d, j = c - i * d;
     const int mp = st->mcur[i];
-    p.X[c] = ddiv(p.H[(long long)mp * d + j], (double)p.nL[mp]);
+    p.X[c] = ddiv(dmul((double)p.Hq[(long long)mp * d + j], p.iscale[j]), (double)p.nL[mp]);
   }
   __threadfence_block();
   __syncthreads();
   zscore_select(p.X, p.k, d, p.l, p.Z, p.dmask, p.dlist, st->nD);
-  // trace
   const int it = st->iterations;
   if (p.tr.cap > 0 && it < p.tr.cap) {
     for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
@@ -607,12 +791,20 @@ __device__ void tail_locality(const RunParams& p) {
 __device__ void tail_assign(const RunParams& p) {
   DevState* st = p.st;
   const int d = p.d;
+  __shared__ long long sz_s[KMAX];
+  if (threadIdx.x < p.k) {
+    sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
+    st->sizes[threadIdx.x] = sz_s[threadIdx.x];
+  }
+  __syncthreads();
   for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
     const int i = c / d, t = c - i * d;
-    const long long sz = p.redc[i];
-    p.mu[c] = (t < st->nD[i] && sz > 0) ? ddiv(p.red[c], (double)sz) : 0.0;
+    const long long sz = sz_s[i];
+    const long long v = take_acc(p, c);
+    double m = 0.0;
+    if (t < st->nD[i] && sz > 0) m = ddiv(dmul((double)v, p.iscale[p.dlist[c]]), (double)sz);
+    p.mu[c] = m;
   }
-  if (threadIdx.x < p.k) st->sizes[threadIdx.x] = p.redc[threadIdx.x];
   __syncthreads();
 }
 
@@ -624,6 +816,16 @@ __device__ void tail_cost(const RunParams& p) {
   DevState* st = p.st;
   const int k = p.k, d = p.d;
   __shared__ int done_s;
+  __shared__ unsigned bad_s;
+  __shared__ int np_s;
+  double* dev = p.Z;  // scratch [k][d]: sum_{p in C_i} |x_pj - mu_ij|
+  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+    const int i = c / d, t = c - i * d;
+    const long long v = take_acc(p, c);
+    dev[c] = (t < st->nD[i]) ? dmul((double)v, p.iscale[p.dlist[c]]) : 0.0;
+  }
+  __threadfence_block();
+  __syncthreads();
   if (threadIdx.x == 0) {
     double cost = 0.0;
     for (int i = 0; i < k; ++i) {
@@ -631,7 +833,7 @@ __device__ void tail_cost(const RunParams& p) {
       if (c == 0) continue;
       double w = 0.0;
       const int nd = st->nD[i];
-      for (int t = 0; t < nd; ++t) w = dadd(w, ddiv(p.red[i * d + t], (double)c));
+      for (int t = 0; t < nd; ++t) w = dadd(w, ddiv(dev[i * d + t], (double)c));
       w = ddiv(w, (double)nd);
       cost = dadd(cost, dmul((double)c, w));
     }
@@ -652,7 +854,6 @@ __device__ void tail_cost(const RunParams& p) {
       st->best_buf = st->cur_buf;
       st->cur_buf ^= 1;
     }
-    // ComputeBadMedoids from MBest
     unsigned bad = 0u;
     const double thr = dmul(ddiv((double)p.n_total, (double)k), p.minDev);
     int smallest = 0;
@@ -661,6 +862,7 @@ __device__ void tail_cost(const RunParams& p) {
       if (st->sizes_best[i] < st->sizes_best[smallest]) smallest = i;
     }
     if (!bad) bad = 1u << smallest;
+    bad_s = bad;
     if (p.tr.cap > 0 && it < p.tr.cap) {
       if (p.tr.cost) p.tr.cost[it] = cost;
       if (p.tr.improved) p.tr.improved[it] = (unsigned char)improved;
@@ -669,18 +871,34 @@ __device__ void tail_cost(const RunParams& p) {
         if (p.tr.bad) p.tr.bad[it * k + i] = (bad >> i) & 1u;
       }
     }
-    // replacement: MCur = MBest with bad slots drawn from M \ MBest
-    int np = 0;
-    for (int t = 0; t < p.nM; ++t) {
-      bool inb = false;
-      for (int i = 0; i < k; ++i) inb |= (st->mbest[i] == t);
-      if (!inb) p.pool[np++] = t;
-    }
     for (int i = 0; i < k; ++i) st->mcur[i] = st->mbest[i];
+  }
+  __threadfence_block();
+  __syncthreads();
+  // pool = ascending positions of M not in MBest (warp compaction)
+  if (threadIdx.x < 32) {
+    int base = 0;
+    for (int t0 = 0; t0 < p.nM; t0 += 32) {
+      const int t = t0 + threadIdx.x;
+      bool inb = t >= p.nM;
+      if (!inb)
+        for (int i = 0; i < k; ++i) inb |= (st->mbest[i] == t);
+      const unsigned b = __ballot_sync(0xffffffffu, !inb);
+      if (!inb) p.pool[base + __popc(b & ((1u << threadIdx.x) - 1u))] = t;
+      base += __popc(b);
+    }
+    if (threadIdx.x == 0) np_s = base;
+  }
+  __threadfence_block();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    // replacement draws (stream IT): the r-th remaining pool entry, in order
+    const unsigned bad = bad_s;
+    int np = np_s;
     unsigned long long rng = st->rng;
     for (int i = 0; i < k; ++i) {
       if (!((bad >> i) & 1u) || np == 0) continue;
-      int r = (int)sm64_uniform(&rng, (unsigned long long)np);
+      const int r = (int)sm64_uniform(&rng, (unsigned long long)np);
       st->mcur[i] = p.pool[r];
       for (int t = r; t + 1 < np; ++t) p.pool[t] = p.pool[t + 1];
       --np;
@@ -688,6 +906,8 @@ __device__ void tail_cost(const RunParams& p) {
     st->rng = rng;
     st->done = (st->itr >= p.itrPat || st->iterations >= p.max_iter) ? 1 : 0;
     done_s = st->done;
+    if (p.use_cond)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, st->done ? 0u : 1u);
   }
   __threadfence_block();
   __syncthreads();
@@ -700,10 +920,14 @@ __device__ void tail_cost(const RunParams& p) {
 __device__ void tail_refine(const RunParams& p) {
   DevState* st = p.st;
   const int k = p.k, d = p.d;
+  __shared__ long long sz_s[KMAX];
+  if (threadIdx.x < k) sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
+  __syncthreads();
   for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d;
-    const long long sz = p.redc[i];
-    p.X[c] = sz > 0 ? ddiv(p.red[c], (double)sz) : 0.0;
+    const int i = c / d, j = c - i * d;
+    const long long sz = sz_s[i];
+    const long long v = take_acc(p, c);
+    p.X[c] = sz > 0 ? ddiv(dmul((double)v, p.iscale[j]), (double)sz) : 0.0;
   }
   __threadfence_block();
   __syncthreads();
@@ -717,7 +941,7 @@ __device__ void tail_refine(const RunParams& p) {
       double s = 0.0;
       for (int t = 0; t < nd; ++t)
         s = dadd(s, fabs(dsub(p.med[(long long)i * d + dl[t]], p.med[(long long)j * d + dl[t]])));
-      double q = ddiv(s, (double)nd);
+      const double q = ddiv(s, (double)nd);
       if (q < m) m = q;
     }
     p.Delta[i] = m;
@@ -725,387 +949,556 @@ __device__ void tail_refine(const RunParams& p) {
   __syncthreads();
 }
 
-// ============================================================ pass kernels
-// Per-point segmental distances to every medoid over D_i (Alg 5 l.4) and the
-// argmin with ties to the smallest i (reading R8), in the oracle's exact
-// fp64 expression.  The fast path compares s_i * (1/|D_i|); only when the
-// runner-up is within 1e-14 relative are the correctly rounded quotients
-// s_i / |D_i| formed and compared.
-__device__ __forceinline__ int assign_point(const double* __restrict__ x, int xs_stride,
-                                            const double* __restrict__ med,
-                                            const int* __restrict__ dl,
-                                            const int* __restrict__ nD,
-                                            const double* __restrict__ rcp, int k,
-                                            int d) {
-  double best = CUDART_INF, second = CUDART_INF;
-  int bi = 0;
-  for (int i = 0; i < k; ++i) {
-    const int nd = nD[i];
-    const int* L = dl + i * d;
-    const double* m = med + i * d;
-    double s = 0.0;
-    for (int t = 0; t < nd; ++t) {
-      const int j = L[t];
-      s = dadd(s, fabs(dsub(x[j * xs_stride], m[j])));
-    }
-    const double q = dmul(s, rcp[i]);
-    if (q < best) {
-      second = best;
-      best = q;
-      bi = i;
-    } else if (q < second) {
-      second = q;
-    }
+// ============================================================ certified tests
+// The fp32 value f approximates the oracle's fp64 value v with
+// |f - v| <= G * v (G from the error analysis of the fp32 evaluation,
+// DESIGN.md section 5).  Returns 1 if v <= T for sure, 0 if v > T for sure,
+// -1 if undecided (tiny or huge values are always undecided).
+__device__ __forceinline__ int cert_le(float f, double T, double G) {
+  const double fd = (double)f;
+  if (!(fd >= 1e-30) || !(T >= 1e-30) || !(fd < 1e30)) return -1;
+  if (fd < T * (1.0 - G)) return 1;
+  if (fd > T * (1.0 + G)) return 0;
+  return -1;
+}
+
+// fp32 approximation of the full-space distance of one staged point (stride P).
+__device__ __forceinline__ float approx_full(const float* __restrict__ x, int P,
+                                             const float* __restrict__ m, int d, int metric) {
+  float s = 0.f;
+  if (metric == 1) {
+    for (int j = 0; j < d; ++j) s += fabsf(x[j * P] - m[j]);
+    return s;
   }
-  if (second > dmul(best, 1.0 + 1e-14)) return bi;
-  // near tie: exact quotients
-  best = CUDART_INF;
-  bi = 0;
+  for (int j = 0; j < d; ++j) {
+    const float t = x[j * P] - m[j];
+    s = fmaf(t, t, s);
+  }
+  return sqrtf(s);
+}
+// same with the point in registers (d <= DREG)
+__device__ __forceinline__ float approx_full_reg(const float (&x)[DREG],
+                                                 const float* __restrict__ m, int d, int metric) {
+  float s = 0.f;
+  if (metric == 1) {
+#pragma unroll
+    for (int j = 0; j < DREG; ++j)
+      if (j < d) s += fabsf(x[j] - m[j]);
+    return s;
+  }
+#pragma unroll
+  for (int j = 0; j < DREG; ++j)
+    if (j < d) {
+      const float t = x[j] - m[j];
+      s = fmaf(t, t, s);
+    }
+  return sqrtf(s);
+}
+
+// Exact (oracle) argmin of seg_{D_i}(x, m_i) = (sum_{j in D_i} |x_j - m_ij|)/|D_i|
+// with ties to the smallest i (Alg 5, reading R8), fp64 from fp32 inputs.
+// sq (may be null) receives every quotient.
+__device__ __noinline__ int exact_argmin(const float* __restrict__ x, int P,
+                                         const float* __restrict__ med32,
+                                         const int* __restrict__ dl, const int* __restrict__ nD,
+                                         int k, int d, const double* __restrict__ Dl,
+                                         int* outside) {
+  double best = CUDART_INF;
+  int bi = 0, out = 1;
   for (int i = 0; i < k; ++i) {
     const int nd = nD[i];
-    const int* L = dl + i * d;
-    const double* m = med + i * d;
     double s = 0.0;
     for (int t = 0; t < nd; ++t) {
-      const int j = L[t];
-      s = dadd(s, fabs(dsub(x[j * xs_stride], m[j])));
+      const int j = dl[i * d + t];
+      s = dadd(s, fabs(dsub((double)x[j * P], (double)med32[i * d + j])));
     }
     const double q = ddiv(s, (double)nd);
+    if (Dl && !(q > Dl[i])) out = 0;
     if (q < best) {
       best = q;
       bi = i;
     }
   }
+  if (outside) *outside = out;
   return bi;
 }
 
+// ============================================================ pass kernels
+// Block = NW consumer warps + 1 producer warp.  Consumer warp w owns the
+// sub-chunk of 32*PPT points starting at q0 = w*32*PPT of every chunk.
+__device__ __forceinline__ long long chunks_of_block(const RunParams& p) {
+  return (p.nchunks > blockIdx.x) ? (p.nchunks - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+}
+
+// Cells (i, t < |D_i|) in cluster order: exclusive scan of |D_i| by warp 0,
+// then a parallel fill.  dl_s[i*d+t] is the dimension, ctr_s[i*d+t] the
+// centre (null: 0).  Returns the number of cells (after a block barrier).
+__device__ int build_cells(Cell* cells, const int* nD_s, int k, int d, int* off_s,
+                           const int* dl_s, const double* ctr_s) {
+  if (threadIdx.x < 32) {
+    const int v = (int)threadIdx.x < k ? nD_s[threadIdx.x] : 0;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if ((int)threadIdx.x >= o) x += y;
+    }
+    if ((int)threadIdx.x < k) off_s[threadIdx.x] = x - v;
+    if (threadIdx.x == 31) off_s[KMAX] = x;
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i])
+      cells[off_s[i] + t] = Cell{i, dl_s[e], e, ctr_s ? ctr_s[e] : 0.0};
+  }
+  __syncthreads();
+  return off_s[KMAX];
+}
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
-__global__ void __launch_bounds__(256) k_locality(RunParams p) {
+// One point per lane; the cached Dist rows of the active slots arrive through
+// the same TMA ring as the data (rows d..).
+template <bool XREG>
+__global__ void __launch_bounds__(288) k_locality(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int P = p.P, d = p.d, k = p.k;
+  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int na = st->n_act;
+  const int ncap = k * d;
   Carve cv(smraw);
-  double* x_s = cv.take<double>((size_t)d * (P + 1));
-  double* med_s = cv.take<double>((size_t)k * d);
-  double* acc_s = cv.take<double>((size_t)k * d);
-  long long* cacc_s = cv.take<long long>(KMAX);
+  Pipe R = carve_pipe(cv, p, d + k, false);
+  float* med_s = cv.take<float>((size_t)k * d);
   ActSlot* act_s = cv.take<ActSlot>(KMAX);
-  ListScratch ls = carve_lists(cv, KMAX * P);
-  const int tid = threadIdx.x;
+  int* row_s = cv.take<int>(KMAX);
+  double* scale_s = cv.take<double>(d);
+  Cell* cells = cv.take<Cell>((size_t)ncap);
+  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX);
+  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
+  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
+  ExtraRows* ex = cv.take<ExtraRows>(1);
+  const long long nmy = chunks_of_block(p);
+  const double G = (double)(d + 8) * 5.9604644775390625e-08;  // (d+8) 2^-24
 
-  for (int a = tid; a < na; a += blockDim.x) act_s[a] = st->act[a];
+  for (int a = threadIdx.x; a < na; a += blockDim.x) act_s[a] = st->act[a];
+  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
+  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  pipe_init(p, R, nw);
   __syncthreads();
-  for (int e = tid; e < na * d; e += blockDim.x) {
-    const int a = e / d, j = e - a * d;
-    med_s[e] = p.med[(long long)act_s[a].slot * d + j];
-    acc_s[e] = 0.0;
+  if (threadIdx.x < 32) {  // rows of the cached slots (warp ballot scan)
+    const int a = threadIdx.x;
+    const bool cached = a < na && !act_s[a].compute;
+    const unsigned b = __ballot_sync(0xffffffffu, cached);
+    const int r = __popc(b & ((1u << a) - 1u));
+    if (a < na) row_s[a] = cached ? d + r : -1;
+    if (cached) ex->src[r] = p.dist + (size_t)act_s[a].mpos * p.n_pad;
+    if (a == 0) ex->n = __popc(b);
   }
-  for (int a = tid; a < KMAX; a += blockDim.x) cacc_s[a] = 0;
+  for (int e = threadIdx.x; e < na * d; e += blockDim.x) {
+    const int a = e / d, j = e - a * d;
+    const float m = p.mrows[(long long)act_s[a].mpos * d + j];
+    med_s[e] = m;
+    cells[e] = Cell{a, j, e, (double)m};
+  }
   __syncthreads();
-
+  long long nfb = 0;
   if (na > 0) {
-    for (long long ch = blockIdx.x; ch < p.nchunks; ch += gridDim.x) {
-      const long long base = ch * P;
-      stage_chunk(p.xs, p.n_pad, d, base, P, x_s);
-      __syncthreads();
-      const long long gp = base + tid;
-      unsigned mask = 0u;
-      if (gp < p.n) {
-        const double* xp = x_s + tid;
+    if (w == nw) {
+      pipe_produce(p, R, nmy, nullptr, ex);
+    } else {
+      unsigned* bal = bal_s + w * KMAX;
+      long long* acc = acc_s + (size_t)w * ncap;
+      const int q = w * 32 + lane;
+      for (long long i = 0; i < nmy; ++i) {
+        const int stg = (int)(i % p.stages);
+        const long long gp = (blockIdx.x + i * gridDim.x) * (long long)P + q;
+        mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+        const float* xs = R.buf + (size_t)stg * R.rows * P;
+        const bool valid = gp < p.n;
+        float xr[DREG];
+        if (XREG) {
+#pragma unroll
+          for (int j = 0; j < DREG; ++j) xr[j] = (j < d) ? xs[j * P + q] : 0.f;
+        }
         for (int a = 0; a < na; ++a) {
           const ActSlot A = act_s[a];
-          float* drow = p.dist + (long long)A.mpos * p.n_pad + gp;
-          bool in;
-          if (A.compute) {  // compute distances only once
-            const double dv = full_dist(xp, P + 1, med_s + a * d, d, p.metric);
-            *drow = __double2float_rn(dv);
-            in = (dv > A.lo) && (dv <= A.hi);
-          } else {  // cached fp32 row: certified decision, exact fallback
-            const float f = __ldg(drow);
-            const int rhi = (f < A.hi32) ? 1 : ((f > A.hi32) ? 0 : -1);
-            const int rlo = (A.lo == -CUDART_INF) ? 1
-                            : (f > A.lo32)        ? 1
-                            : (f < A.lo32)        ? 0
-                                                  : -1;
-            if (rhi == 0 || rlo == 0) {
-              in = false;
-            } else if (rhi == 1 && rlo == 1) {
-              in = true;
+          bool in = false;
+          if (valid) {
+            float f;
+            if (A.compute) {  // compute distances only once
+              f = XREG ? approx_full_reg(xr, med_s + a * d, d, p.metric)
+                       : approx_full(xs + q, P, med_s + a * d, d, p.metric);
+              p.dist[(long long)A.mpos * p.n_pad + gp] = f;
             } else {
-              const double dv = full_dist(xp, P + 1, med_s + a * d, d, p.metric);
+              f = xs[row_s[a] * P + q];
+            }
+            const int rhi = cert_le(f, A.hi, G);
+            const int rlo = (A.lo == -CUDART_INF) ? 0 : cert_le(f, A.lo, G);
+            if (rhi >= 0 && rlo >= 0) {
+              in = (rhi == 1) && (rlo == 0);  // v <= hi and not v <= lo
+            } else {
+              const double dv = full_dist(xs + q, P, med_s + a * d, d, p.metric);
               in = (dv > A.lo) && (dv <= A.hi);
+              ++nfb;
             }
           }
-          if (in) mask |= 1u << a;
+          put_ballot(bal, a, in);
         }
+        __syncwarp();
+        if (lane < na) cnt_s[w * KMAX + lane] += __popc(bal[lane]);
+        // cells (a, j): band sum of |x_j - m_aj| (eq 6)
+        warp_cells<1, 1>(xs, P, w * 32, cells, na * d, bal, acc, scale_s);
+        pipe_release(R, stg);
       }
-      build_lists(mask, na, ls);
-      // cells (a, j): sum over the band of |x_j - m_aj| (eq 6)
-      for (int c = tid; c < na * d; c += blockDim.x) {
-        const int a = c / d, j = c - a * d;
-        const int cnt = ls.cnt[a];
-        if (cnt == 0) continue;
-        acc_s[c] = dadd(acc_s[c], list_sum<1>(x_s + j * (P + 1), ls.list + ls.base[a],
-                                              cnt, med_s[c]));
-      }
-      if (tid < na) cacc_s[tid] += ls.cnt[tid];
-      __syncthreads();
     }
   }
-  // per-block partials
-  const int stride = k * d;
-  for (int c = tid; c < na * d; c += blockDim.x)
-    p.part[(long long)blockIdx.x * stride + c] = acc_s[c];
-  for (int a = tid; a < KMAX; a += blockDim.x)
-    p.partc[(long long)blockIdx.x * KMAX + a] = cacc_s[a];
+  __syncthreads();
+  flush_warps(p, acc_s, nw, ncap, na * d, cnt_s, na);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[0], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[0])) return;
-  reduce_partials(p.part, p.partc, gridDim.x, stride, na * d, na, p.red, p.redc);
+  const unsigned long long t0 = gtimer();
   tail_locality(p);
+  if (threadIdx.x == 0) st->tail_ns[0] += gtimer() - t0;
 }
 
 // --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8).
-__global__ void __launch_bounds__(256) k_assign(RunParams p) {
+// PPT points per lane so every term-table entry loaded serves PPT points.
+struct Term {
+  int joff;  // j * P
+  float m;   // m_ij
+};
+
+template <int PPT>
+__global__ void __launch_bounds__(160) k_assign(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int P = p.P, d = p.d, k = p.k;
+  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ncap = k * d;
   Carve cv(smraw);
-  double* x_s = cv.take<double>((size_t)d * (P + 1));
-  double* med_s = cv.take<double>((size_t)k * d);
-  double* acc_s = cv.take<double>((size_t)k * d);
-  long long* cacc_s = cv.take<long long>(KMAX);
+  Pipe R = carve_pipe(cv, p, d, false);
+  float* med_s = cv.take<float>((size_t)k * d);
+  Term* tab_s = cv.take<Term>((size_t)k * d);
   int* dl_s = cv.take<int>((size_t)k * d);
   int* nD_s = cv.take<int>(KMAX);
-  double* rcp_s = cv.take<double>(KMAX);
-  ListScratch ls = carve_lists(cv, P);
-  const int tid = threadIdx.x;
+  int* off_s = cv.take<int>(KMAX + 1);
+  float* rcp_s = cv.take<float>(KMAX);
+  double* scale_s = cv.take<double>(d);
+  Cell* cells = cv.take<Cell>((size_t)ncap);
+  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX * PPT);
+  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
+  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
   unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  const long long nmy = chunks_of_block(p);
 
-  for (int e = tid; e < k * d; e += blockDim.x) {
-    med_s[e] = p.med[e];
-    dl_s[e] = p.dlist[e];
-    acc_s[e] = 0.0;
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    nD_s[i] = st->nD[i];
+    rcp_s[i] = 1.0f / (float)st->nD[i];
   }
-  for (int i = tid; i < KMAX; i += blockDim.x) {
-    cacc_s[i] = 0;
-    if (i < k) {
-      nD_s[i] = st->nD[i];
-      rcp_s[i] = ddiv(1.0, (double)st->nD[i]);
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
+    dl_s[e] = p.dlist[e];
+  }
+  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
+  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  pipe_init(p, R, nw);
+  __syncthreads();
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i]) {
+      const int j = dl_s[e];
+      tab_s[e].joff = j * P;
+      tab_s[e].m = med_s[i * d + j];
+    }
+  }
+  const int ncell = build_cells(cells, nD_s, k, d, off_s, dl_s, nullptr);
+  int ndmax = 0;
+  for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
+  const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
+  long long nfb = 0;
+  if (w == nw) {
+    pipe_produce(p, R, nmy, nullptr, nullptr);
+  } else {
+    unsigned* bal = bal_s + w * KMAX * PPT;
+    long long* acc = acc_s + (size_t)w * ncap;
+    const int q0 = w * 32 * PPT;
+    for (long long i = 0; i < nmy; ++i) {
+      const int stg = (int)(i % p.stages);
+      const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
+      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+      const float* xs = R.buf + (size_t)stg * R.rows * P;
+      const float* xq = xs + q0 + lane;
+      float best[PPT], second[PPT];
+      int bi[PPT];
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) {
+        best[u] = CUDART_INF_F;
+        second[u] = CUDART_INF_F;
+        bi[u] = 0;
+      }
+      for (int c = 0; c < k; ++c) {
+        const int nd = nD_s[c];
+        const Term* tb = tab_s + c * d;
+        // fp32 partial sums in any order: the certified bound only needs the
+        // number of terms; 4 terms in flight per point
+        float s[PPT], s2[PPT];
+#pragma unroll
+        for (int u = 0; u < PPT; ++u) {
+          s[u] = 0.f;
+          s2[u] = 0.f;
+        }
+        int t = 0;
+        for (; t + 4 <= nd; t += 4) {
+          const Term e0 = tb[t], e1 = tb[t + 1], e2 = tb[t + 2], e3 = tb[t + 3];
+#pragma unroll
+          for (int u = 0; u < PPT; ++u) {
+            const float* xu = xq + u * 32;
+            const float a0 = fabsf(xu[e0.joff] - e0.m), a1 = fabsf(xu[e1.joff] - e1.m);
+            const float a2 = fabsf(xu[e2.joff] - e2.m), a3 = fabsf(xu[e3.joff] - e3.m);
+            s[u] += a0 + a1;
+            s2[u] += a2 + a3;
+          }
+        }
+        for (; t < nd; ++t) {
+          const Term e = tb[t];
+#pragma unroll
+          for (int u = 0; u < PPT; ++u) s[u] += fabsf(xq[u * 32 + e.joff] - e.m);
+        }
+        const float r = rcp_s[c];
+#pragma unroll
+        for (int u = 0; u < PPT; ++u) {
+          const float qv = (s[u] + s2[u]) * r;
+          if (qv < best[u]) {
+            second[u] = best[u];
+            best[u] = qv;
+            bi[u] = c;
+          } else if (qv < second[u]) {
+            second[u] = qv;
+          }
+        }
+      }
+      int lbl[PPT];
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) {
+        const int q = q0 + u * 32 + lane;
+        const long long gp = base + q;
+        lbl[u] = -1;
+        if (gp >= p.n) continue;
+        const double b = (double)best[u], s2v = (double)second[u];
+        const bool certain =
+            (b >= 1e-30) && (s2v < 1e30) && (s2v * (1.0 - G) > b * (1.0 + G));
+        lbl[u] = bi[u];
+        if (!certain) {
+          lbl[u] = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
+          ++nfb;
+        }
+        lab[gp] = (unsigned char)lbl[u];
+      }
+      for (int c = 0; c < k; ++c)
+#pragma unroll
+        for (int u = 0; u < PPT; ++u) put_ballot(bal, c * PPT + u, lbl[u] == c);
+      __syncwarp();
+      if (lane < k) {
+        int cn = 0;
+#pragma unroll
+        for (int u = 0; u < PPT; ++u) cn += __popc(bal[lane * PPT + u]);
+        cnt_s[w * KMAX + lane] += cn;
+      }
+      warp_cells<0, PPT>(xs, P, q0, cells, ncell, bal, acc, scale_s);
+      pipe_release(R, stg);
     }
   }
   __syncthreads();
-  for (long long ch = blockIdx.x; ch < p.nchunks; ch += gridDim.x) {
-    const long long base = ch * P;
-    stage_chunk(p.xs, p.n_pad, d, base, P, x_s);
-    __syncthreads();
-    const long long gp = base + tid;
-    unsigned mask = 0u;
-    if (gp < p.n) {
-      const int bi = assign_point(x_s + tid, P + 1, med_s, dl_s, nD_s, rcp_s, k, d);
-      lab[gp] = (unsigned char)bi;
-      mask = 1u << bi;
-    }
-    build_lists(mask, k, ls);
-    for (int c = tid; c < k * d; c += blockDim.x) {
-      const int i = c / d, t = c - i * d;
-      const int cnt = ls.cnt[i];
-      if (t >= nD_s[i] || cnt == 0) continue;
-      const int j = dl_s[c];
-      acc_s[c] = dadd(acc_s[c], list_sum<0>(x_s + j * (P + 1), ls.list + ls.base[i], cnt, 0.0));
-    }
-    if (tid < k) cacc_s[tid] += ls.cnt[tid];
-    __syncthreads();
-  }
-  const int stride = k * d;
-  for (int c = tid; c < stride; c += blockDim.x)
-    p.part[(long long)blockIdx.x * stride + c] = acc_s[c];
-  for (int a = tid; a < KMAX; a += blockDim.x)
-    p.partc[(long long)blockIdx.x * KMAX + a] = cacc_s[a];
+  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, k);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[1])) return;
-  reduce_partials(p.part, p.partc, gridDim.x, stride, stride, k, p.red, p.redc);
+  const unsigned long long t0 = gtimer();
   tail_assign(p);
+  if (threadIdx.x == 0) st->tail_ns[1] += gtimer() - t0;
 }
 
-// --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) + control tail.
-__global__ void __launch_bounds__(256) k_cost(RunParams p) {
+// --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) + control tail, and the
+// refinement X over CBest (Alg 1 l.16-17) which has the same shape.
+// REF = 0: cells (i, t) over D_i of |x - mu_i|, labels of the current buffer.
+// REF = 1: cells (i, j) over all d of |x - mbest_ij|, labels of CBest.
+template <int REF>
+__global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
   DevState* st = p.st;
-  if (st->done) return;
+  if (!REF && st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int P = p.P, d = p.d, k = p.k;
+  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ncap = k * d;
   Carve cv(smraw);
-  double* x_s = cv.take<double>((size_t)d * (P + 1));
-  double* mu_s = cv.take<double>((size_t)k * d);
-  double* acc_s = cv.take<double>((size_t)k * d);
+  Pipe R = carve_pipe(cv, p, d, true);
+  double* ctr_s = cv.take<double>((size_t)k * d);
   int* dl_s = cv.take<int>((size_t)k * d);
   int* nD_s = cv.take<int>(KMAX);
-  ListScratch ls = carve_lists(cv, P);
-  const int tid = threadIdx.x;
-  const unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
-
-  for (int e = tid; e < k * d; e += blockDim.x) {
-    mu_s[e] = p.mu[e];
-    dl_s[e] = p.dlist[e];
-    acc_s[e] = 0.0;
+  int* off_s = cv.take<int>(KMAX + 1);
+  double* scale_s = cv.take<double>(d);
+  Cell* cells = cv.take<Cell>((size_t)ncap);
+  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX);
+  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
+  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
+  const unsigned char* lab =
+      REF ? (st->best_buf ? p.lab1 : p.lab0) : (st->cur_buf ? p.lab1 : p.lab0);
+  const long long nmy = chunks_of_block(p);
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    ctr_s[e] = REF ? (double)p.mrows[(long long)st->mbest[i] * d + (e - i * d)] : p.mu[e];
+    dl_s[e] = REF ? e - i * d : p.dlist[e];
   }
-  for (int i = tid; i < k; i += blockDim.x) nD_s[i] = st->nD[i];
+  for (int i = threadIdx.x; i < k; i += blockDim.x) nD_s[i] = REF ? d : st->nD[i];
+  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
+  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  pipe_init(p, R, nw);
   __syncthreads();
-  for (long long ch = blockIdx.x; ch < p.nchunks; ch += gridDim.x) {
-    const long long base = ch * P;
-    stage_chunk(p.xs, p.n_pad, d, base, P, x_s);
-    const long long gp = base + tid;
-    const unsigned mask = (gp < p.n) ? (1u << lab[gp]) : 0u;
-    __syncthreads();
-    build_lists(mask, k, ls);
-    for (int c = tid; c < k * d; c += blockDim.x) {
-      const int i = c / d, t = c - i * d;
-      const int cnt = ls.cnt[i];
-      if (t >= nD_s[i] || cnt == 0) continue;
-      const int j = dl_s[c];
-      acc_s[c] = dadd(acc_s[c], list_sum<1>(x_s + j * (P + 1), ls.list + ls.base[i], cnt,
-                                            mu_s[c]));
+  const int ncell = build_cells(cells, nD_s, k, d, off_s, dl_s, ctr_s);
+  if (w == nw) {
+    pipe_produce(p, R, nmy, lab, nullptr);
+  } else {
+    unsigned* bal = bal_s + w * KMAX;
+    long long* acc = acc_s + (size_t)w * ncap;
+    const int q = w * 32 + lane;
+    for (long long i = 0; i < nmy; ++i) {
+      const int stg = (int)(i % p.stages);
+      const long long gp = (blockIdx.x + i * gridDim.x) * (long long)P + q;
+      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+      const float* xs = R.buf + (size_t)stg * R.rows * P;
+      const int lb = gp < p.n ? (int)R.lab[(size_t)stg * P + q] : -1;
+      for (int c = 0; c < k; ++c) put_ballot(bal, c, lb == c);
+      __syncwarp();
+      if (REF && lane < k) cnt_s[w * KMAX + lane] += __popc(bal[lane]);
+      warp_cells<1, 1>(xs, P, w * 32, cells, ncell, bal, acc, scale_s);
+      pipe_release(R, stg);
     }
-    __syncthreads();
   }
-  const int stride = k * d;
-  for (int c = tid; c < stride; c += blockDim.x)
-    p.part[(long long)blockIdx.x * stride + c] = acc_s[c];
-  if (!p.fuse_tail) return;
-  if (!last_block(&st->ticket[2])) return;
-  reduce_partials(p.part, p.partc, gridDim.x, stride, stride, 0, p.red, p.redc);
-  tail_cost(p);
-}
-
-// --- Refinement X over CBest (Alg 1 l.16-17): sums of |x_j - mbest_ij| for
-// every dimension over each best cluster.  p.med holds the MBest rows.
-__global__ void __launch_bounds__(256) k_refine_x(RunParams p) {
-  DevState* st = p.st;
-  extern __shared__ __align__(16) unsigned char smraw[];
-  const int P = p.P, d = p.d, k = p.k;
-  Carve cv(smraw);
-  double* x_s = cv.take<double>((size_t)d * (P + 1));
-  double* med_s = cv.take<double>((size_t)k * d);
-  double* acc_s = cv.take<double>((size_t)k * d);
-  long long* cacc_s = cv.take<long long>(KMAX);
-  ListScratch ls = carve_lists(cv, P);
-  const int tid = threadIdx.x;
-  const unsigned char* lab = st->best_buf ? p.lab1 : p.lab0;
-  for (int e = tid; e < k * d; e += blockDim.x) {
-    const int i = e / d, j = e - i * d;
-    med_s[e] = (double)p.mrows[(long long)st->mbest[i] * d + j];
-    acc_s[e] = 0.0;
-  }
-  for (int a = tid; a < KMAX; a += blockDim.x) cacc_s[a] = 0;
   __syncthreads();
-  for (long long ch = blockIdx.x; ch < p.nchunks; ch += gridDim.x) {
-    const long long base = ch * P;
-    stage_chunk(p.xs, p.n_pad, d, base, P, x_s);
-    const long long gp = base + tid;
-    const unsigned mask = (gp < p.n) ? (1u << lab[gp]) : 0u;
-    __syncthreads();
-    build_lists(mask, k, ls);
-    for (int c = tid; c < k * d; c += blockDim.x) {
-      const int i = c / d, j = c - i * d;
-      const int cnt = ls.cnt[i];
-      if (cnt == 0) continue;
-      acc_s[c] = dadd(acc_s[c], list_sum<1>(x_s + j * (P + 1), ls.list + ls.base[i], cnt,
-                                            med_s[c]));
-    }
-    if (tid < k) cacc_s[tid] += ls.cnt[tid];
-    __syncthreads();
-  }
-  const int stride = k * d;
-  for (int c = tid; c < stride; c += blockDim.x)
-    p.part[(long long)blockIdx.x * stride + c] = acc_s[c];
-  for (int a = tid; a < KMAX; a += blockDim.x)
-    p.partc[(long long)blockIdx.x * KMAX + a] = cacc_s[a];
+  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, REF ? k : 0);
   if (!p.fuse_tail) return;
-  if (!last_block(&st->ticket[3])) return;
-  // MBest rows (fp64) for Delta
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) p.med[e] = med_s[e];
-  reduce_partials(p.part, p.partc, gridDim.x, stride, stride, k, p.red, p.redc);
-  tail_refine(p);
+  if (!last_block(&st->ticket[REF ? 3 : 2])) return;
+  const unsigned long long t0 = gtimer();
+  if (REF) {
+    for (int e = threadIdx.x; e < k * d; e += blockDim.x) p.med[e] = ctr_s[e];
+    __threadfence_block();
+    __syncthreads();
+    tail_refine(p);
+  } else {
+    tail_cost(p);
+  }
+  if (threadIdx.x == 0) st->tail_ns[REF ? 3 : 2] += gtimer() - t0;
 }
 
 // --- Final AssignPoints with D* (Alg 1 l.18) and RemoveOutliers (l.19):
 // outlier iff seg_{D*_i}(x, m_i) > Delta_i for every i (reading R17).
-__global__ void __launch_bounds__(256) k_final(RunParams p) {
+template <int PPT>
+__global__ void __launch_bounds__(160) k_final(RunParams p) {
   DevState* st = p.st;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int P = p.P, d = p.d, k = p.k;
+  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   Carve cv(smraw);
-  double* x_s = cv.take<double>((size_t)d * (P + 1));
-  double* med_s = cv.take<double>((size_t)k * d);
+  Pipe R = carve_pipe(cv, p, d, false);
+  float* med_s = cv.take<float>((size_t)k * d);
+  Term* tab_s = cv.take<Term>((size_t)k * d);
   int* dl_s = cv.take<int>((size_t)k * d);
   int* nD_s = cv.take<int>(KMAX);
-  double* rcp_s = cv.take<double>(KMAX);
+  float* rcp_s = cv.take<float>(KMAX);
   double* Dl_s = cv.take<double>(KMAX);
-  const int tid = threadIdx.x;
-  for (int e = tid; e < k * d; e += blockDim.x) {
-    med_s[e] = p.med[e];
-    dl_s[e] = p.dlist[e];
-  }
-  for (int i = tid; i < k; i += blockDim.x) {
+  const long long nmy = chunks_of_block(p);
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
     nD_s[i] = st->nD[i];
-    rcp_s[i] = ddiv(1.0, (double)st->nD[i]);
+    rcp_s[i] = 1.0f / (float)st->nD[i];
     Dl_s[i] = p.Delta[i];
   }
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    med_s[e] = p.mrows[(long long)st->mbest[i] * d + (e - i * d)];
+    dl_s[e] = p.dlist[e];
+  }
+  pipe_init(p, R, nw);
   __syncthreads();
-  for (long long ch = blockIdx.x; ch < p.nchunks; ch += gridDim.x) {
-    const long long base = ch * P;
-    stage_chunk(p.xs, p.n_pad, d, base, P, x_s);
-    __syncthreads();
-    const long long gp = base + tid;
-    if (gp < p.n) {
-      const double* xp = x_s + tid;
-      const int bi = assign_point(xp, P + 1, med_s, dl_s, nD_s, rcp_s, k, d);
-      bool outside_all = true;
-      for (int i = 0; i < k && outside_all; ++i) {
-        const int nd = nD_s[i];
-        double s = 0.0;
-        for (int t = 0; t < nd; ++t) {
-          const int j = dl_s[i * d + t];
-          s = dadd(s, fabs(dsub(xp[j * (P + 1)], med_s[i * d + j])));
-        }
-        const double q = dmul(s, rcp_s[i]);
-        const double D = Dl_s[i];
-        bool gt;
-        if (q > dmul(D, 1.0 + 1e-14))
-          gt = true;
-        else if (q < dmul(D, 1.0 - 1e-14))
-          gt = false;
-        else
-          gt = ddiv(s, (double)nd) > D;
-        outside_all = gt;
-      }
-      p.out_labels[gp] = outside_all ? -1 : bi;
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i]) {
+      const int j = dl_s[e];
+      tab_s[e].joff = j * P;
+      tab_s[e].m = med_s[i * d + j];
     }
-    __syncthreads();
   }
-}
-
-// ============================================================ multi-GPU tails
-__global__ void k_reduce(RunParams p, int tail, int G) {
-  DevState* st = p.st;
-  if (tail != TAIL_REF && st->done) return;
-  const int kd = p.k * p.d;
-  int ncell = kd, ncnt = p.k;
-  if (tail == TAIL_LOC) {
-    ncell = st->n_act * p.d;
-    ncnt = st->n_act;
-  } else if (tail == TAIL_COST) {
-    ncnt = 0;
-  }
-  // unused entries are zeroed so a full-length allreduce is exact
-  for (int c = threadIdx.x; c < kd; c += blockDim.x) p.red[c] = 0.0;
-  for (int c = threadIdx.x; c < KMAX; c += blockDim.x) p.redc[c] = 0;
   __syncthreads();
-  reduce_partials(p.part, p.partc, G, kd, ncell, ncnt, p.red, p.redc);
+  int ndmax = 0;
+  for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
+  const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
+  long long nfb = 0;
+  if (w == nw) {
+    pipe_produce(p, R, nmy, nullptr, nullptr);
+  } else {
+    const int q0 = w * 32 * PPT;
+    for (long long i = 0; i < nmy; ++i) {
+      const int stg = (int)(i % p.stages);
+      const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
+      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+      const float* xs = R.buf + (size_t)stg * R.rows * P;
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) {
+        const int q = q0 + u * 32 + lane;
+        const long long gp = base + q;
+        if (gp >= p.n) continue;
+        float best = CUDART_INF_F, second = CUDART_INF_F;
+        int bi = 0;
+        int out = 1;        // outside every sphere so far (certainly)
+        int undecided = 0;  // some sphere test needs the exact value
+        for (int c = 0; c < k; ++c) {
+          const int nd = nD_s[c];
+          const Term* tb = tab_s + c * d;
+          float s = 0.f, s2 = 0.f;
+          int t = 0;
+          for (; t + 2 <= nd; t += 2) {
+            s += fabsf(xs[tb[t].joff + q] - tb[t].m);
+            s2 += fabsf(xs[tb[t + 1].joff + q] - tb[t + 1].m);
+          }
+          if (t < nd) s += fabsf(xs[tb[t].joff + q] - tb[t].m);
+          const float qv = (s + s2) * rcp_s[c];
+          if (qv < best) {
+            second = best;
+            best = qv;
+            bi = c;
+          } else if (qv < second) {
+            second = qv;
+          }
+          const int le = cert_le(qv, Dl_s[c], G);  // seg <= Delta_c ?
+          if (le == 1) out = 0;
+          if (le < 0) undecided = 1;
+        }
+        const double b = (double)best, s2v = (double)second;
+        const bool certain =
+            (b >= 1e-30) && (s2v < 1e30) && (s2v * (1.0 - G) > b * (1.0 + G));
+        int lbl = bi;
+        if (!certain || (out && undecided)) {
+          int outx = 0;
+          lbl = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, Dl_s, &outx);
+          if (out && undecided) out = outx;
+          ++nfb;
+        }
+        p.out_labels[gp] = out ? -1 : lbl;
+      }
+      pipe_release(R, stg);
+    }
+  }
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[2], (unsigned long long)nfb);
 }
 
+// ============================================================ multi-GPU tail
 __global__ void k_tail(RunParams p, int tail) {
   DevState* st = p.st;
   if (tail == TAIL_LOC) {
@@ -1122,81 +1515,91 @@ __global__ void k_tail(RunParams p, int tail) {
       const int i = e / p.d, j = e - i * p.d;
       p.med[e] = (double)p.mrows[(long long)st->mbest[i] * p.d + j];
     }
+    __threadfence_block();
     __syncthreads();
     tail_refine(p);
   }
 }
 
-void launch_reduce(const RunParams& p, const PassShape& ps, int tail,
-                   cudaStream_t s) {
-  k_reduce<<<1, 256, 0, s>>>(p, tail, ps.grid);
-}
-
-void launch_tail(const RunParams& p, int tail, cudaStream_t s) {
-  k_tail<<<1, 256, 0, s>>>(p, tail);
-}
+void launch_tail(const RunParams& p, int tail, cudaStream_t s) { k_tail<<<1, 256, 0, s>>>(p, tail); }
 
 // ============================================================ shapes
-static size_t smem_loc(int P, int d, int k) {
-  return carve_size({sizeof(double) * (size_t)d * (P + 1), sizeof(double) * (size_t)k * d,
-                     sizeof(double) * (size_t)k * d, sizeof(long long) * KMAX,
-                     sizeof(ActSlot) * KMAX}) +
-         lists_bytes(KMAX * P);
+// Chunk P = 32 * PPT * NW points.  d <= 32: P = 256 (locality / labelsum 8
+// consumer warps x 1 point per lane, assign / final 4 warps x 2 points);
+// larger d: P = 128 or 64 so that the ring of (d + k) rows stays small.
+static size_t smem_loc(int P, int d, int k, int stages, int nw) {
+  CarveSize cs;
+  size_pipe(cs, d + k, P, stages, false);
+  cs.add<float>((size_t)k * d).add<ActSlot>(KMAX).add<int>(KMAX).add<double>(d);
+  cs.add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX);
+  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX).add<ExtraRows>(1);
+  return cs.s + 64;
 }
-static size_t smem_asg(int P, int d, int k) {
-  return carve_size({sizeof(double) * (size_t)d * (P + 1), sizeof(double) * (size_t)k * d,
-                     sizeof(double) * (size_t)k * d, sizeof(long long) * KMAX,
-                     sizeof(int) * (size_t)k * d, sizeof(int) * KMAX,
-                     sizeof(double) * KMAX}) +
-         lists_bytes(P);
+static size_t smem_asg(int P, int d, int k, int stages, int nw) {
+  CarveSize cs;
+  size_pipe(cs, d, P, stages, false);
+  cs.add<float>((size_t)k * d).add<Term>((size_t)k * d).add<int>((size_t)k * d);
+  cs.add<int>(KMAX).add<int>(KMAX + 1).add<float>(KMAX).add<double>(d);
+  cs.add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX * 2);
+  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX);
+  return cs.s + 64;
 }
-static size_t smem_cost(int P, int d, int k) {
-  return carve_size({sizeof(double) * (size_t)d * (P + 1), sizeof(double) * (size_t)k * d,
-                     sizeof(double) * (size_t)k * d, sizeof(int) * (size_t)k * d,
-                     sizeof(int) * KMAX}) +
-         lists_bytes(P);
+static size_t smem_lsum(int P, int d, int k, int stages, int nw) {
+  CarveSize cs;
+  size_pipe(cs, d, P, stages, true);
+  cs.add<double>((size_t)k * d).add<int>((size_t)k * d).add<int>(KMAX).add<int>(KMAX + 1);
+  cs.add<double>(d).add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX);
+  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX);
+  return cs.s + 64;
 }
-static size_t smem_ref(int P, int d, int k) {
-  return carve_size({sizeof(double) * (size_t)d * (P + 1), sizeof(double) * (size_t)k * d,
-                     sizeof(double) * (size_t)k * d, sizeof(long long) * KMAX}) +
-         lists_bytes(P);
-}
-static size_t smem_fin(int P, int d, int k) {
-  return carve_size({sizeof(double) * (size_t)d * (P + 1), sizeof(double) * (size_t)k * d,
-                     sizeof(int) * (size_t)k * d, sizeof(int) * KMAX,
-                     sizeof(double) * KMAX, sizeof(double) * KMAX});
+static size_t smem_fin(int P, int d, int k, int stages) {
+  CarveSize cs;
+  size_pipe(cs, d, P, stages, false);
+  cs.add<float>((size_t)k * d).add<Term>((size_t)k * d).add<int>((size_t)k * d);
+  cs.add<int>(KMAX).add<float>(KMAX).add<double>(KMAX);
+  return cs.s + 64;
 }
 
 PassShape pass_shape(int d, int k, int num_sms) {
   PassShape ps;
-  int P = PMAX;
-  const size_t budget = 100 * 1024;
-  while (P > 32 && (smem_loc(P, d, k) > budget || smem_asg(P, d, k) > budget)) P >>= 1;
+  int P = 256, stages = 3;
+  const int cfg[6][2] = {{256, 3}, {256, 2}, {128, 3}, {128, 2}, {64, 3}, {64, 2}};
+  for (int c = 0; c < 6; ++c) {
+    P = cfg[c][0];
+    stages = cfg[c][1];
+    if ((size_t)stages * (d + k) * P * 4 <= 60 * 1024) break;
+  }
   ps.P = P;
-  ps.smem_loc = smem_loc(P, d, k);
-  ps.smem_asg = smem_asg(P, d, k);
-  ps.smem_cost = smem_cost(P, d, k);
-  ps.smem_ref = smem_ref(P, d, k);
-  ps.smem_fin = smem_fin(P, d, k);
+  ps.stages = stages;
+  const int nw1 = P / 32, nw2 = P / 64;  // consumer warps at 1 / 2 points per lane
+  ps.tpb_loc = 32 * (nw1 + 1);
+  ps.tpb_asg = 32 * (nw2 + 1);
+  ps.tpb_lsum = 32 * (nw1 + 1);
+  ps.tpb_fin = 32 * (nw2 + 1);
+  ps.smem_loc = smem_loc(P, d, k, stages, nw1);
+  ps.smem_asg = smem_asg(P, d, k, stages, nw2);
+  ps.smem_cost = smem_lsum(P, d, k, stages, nw1);
+  ps.smem_ref = ps.smem_cost;
+  ps.smem_fin = smem_fin(P, d, k, stages);
   size_t mx = ps.smem_loc;
   if (ps.smem_asg > mx) mx = ps.smem_asg;
-  // resident blocks per SM limited by shared memory (228 KB per SM) and by
-  // 2048 threads per SM
-  int by_smem = (int)((228 * 1024) / (mx + 1024));
-  int by_thr = 2048 / P;
-  int per_sm = by_smem < by_thr ? by_smem : by_thr;
+  if (ps.smem_cost > mx) mx = ps.smem_cost;
+  int per_sm = (int)((227 * 1024) / (mx + 1024));
   if (per_sm < 1) per_sm = 1;
+  if (per_sm > 2048 / ps.tpb_loc) per_sm = 2048 / ps.tpb_loc;
   if (per_sm > 8) per_sm = 8;
+  ps.per_sm = per_sm;
   ps.grid = num_sms * per_sm;
   return ps;
 }
 
 cudaError_t configure_kernels(const PassShape& ps) {
   cudaError_t e;
-  const void* fns[] = {(const void*)k_locality, (const void*)k_assign, (const void*)k_cost,
-                       (const void*)k_refine_x, (const void*)k_final};
-  size_t sm[] = {ps.smem_loc, ps.smem_asg, ps.smem_cost, ps.smem_ref, ps.smem_fin};
-  for (int i = 0; i < 5; ++i) {
+  const void* fns[] = {(const void*)k_locality<true>, (const void*)k_locality<false>,
+                       (const void*)k_assign<2>,       (const void*)k_labelsum<0>,
+                       (const void*)k_labelsum<1>,     (const void*)k_final<2>};
+  size_t sm[] = {ps.smem_loc, ps.smem_loc, ps.smem_asg, ps.smem_cost, ps.smem_ref, ps.smem_fin};
+  for (int i = 0; i < 6; ++i) {
     e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm[i]);
     if (e != cudaSuccess) return e;
   }
@@ -1204,19 +1607,22 @@ cudaError_t configure_kernels(const PassShape& ps) {
 }
 
 void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_locality<<<ps.grid, ps.P, ps.smem_loc, s>>>(p);
+  if (p.d <= DREG)
+    k_locality<true><<<ps.grid, ps.tpb_loc, ps.smem_loc, s>>>(p);
+  else
+    k_locality<false><<<ps.grid, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_assign<<<ps.grid, ps.P, ps.smem_asg, s>>>(p);
+  k_assign<2><<<ps.grid, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_cost<<<ps.grid, ps.P, ps.smem_cost, s>>>(p);
+  k_labelsum<0><<<ps.grid, ps.tpb_lsum, ps.smem_cost, s>>>(p);
 }
 void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_refine_x<<<ps.grid, ps.P, ps.smem_ref, s>>>(p);
+  k_labelsum<1><<<ps.grid, ps.tpb_lsum, ps.smem_ref, s>>>(p);
 }
 void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_final<<<ps.grid, ps.P, ps.smem_fin, s>>>(p);
+  k_final<2><<<ps.grid, ps.tpb_fin, ps.smem_fin, s>>>(p);
 }
 
 }  // namespace pc

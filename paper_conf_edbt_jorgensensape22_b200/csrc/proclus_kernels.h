@@ -10,27 +10,31 @@
 namespace pc {
 
 struct PassShape {
-  int P;          // points per chunk == threads per block
-  int grid;       // persistent blocks (multiple of the SM count)
+  int P;          // points per chunk
+  int stages;     // bulk-copy ring depth
+  int tpb_loc, tpb_asg, tpb_lsum, tpb_fin;  // threads per block of each pass
+  int per_sm;     // resident blocks per SM
+  int grid;       // persistent blocks (SM count x per_sm)
   size_t smem_loc, smem_asg, smem_cost, smem_ref, smem_fin;
 };
 
-// N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value.
-void launch_pack_soa(const float* in, long long n, int d, long long n_pad,
-                     float* xs, int* bad, cudaStream_t s);
+// N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value;
+// colmax[j] = max(colmax[j], bits of max |x_j|).
+void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
+                     unsigned* colmax, cudaStream_t s);
 // rows of the given (global) ids; rows outside [row_offset, row_offset+n)
 // are zero (they are filled by another rank and summed by the allreduce).
-void launch_gather_rows(const float* xs, long long n_pad, int d,
-                        const long long* ids, long long row_offset,
-                        long long n_local, int cnt, float* out, cudaStream_t s);
-// Greedy (Alg 2) in one CTA: spos[nM] positions into S.
-cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0,
-                          int metric, int* spos, double* pickdist,
-                          cudaStream_t s);
+void launch_gather_rows(const float* xs, long long n_pad, int d, const long long* ids,
+                        long long row_offset, long long n_local, int cnt, float* out,
+                        cudaStream_t s);
+// Greedy (Alg 2): spos[nM] positions into S.  scratch holds
+// greedy_scratch_doubles(nS) doubles (the #S x #S distance matrix).
+size_t greedy_scratch_doubles(int nS);
+cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
+                          double* scratch, int* spos, double* pickdist, cudaStream_t s);
 // M rows and ids from S rows and positions.
-void launch_gather_m(const float* srows, const long long* sids, const int* spos,
-                     int nM, int d, float* mrows, long long* mids,
-                     cudaStream_t s);
+void launch_gather_m(const float* srows, const long long* sids, const int* spos, int nM, int d,
+                     float* mrows, long long* mids, cudaStream_t s);
 
 PassShape pass_shape(int d, int k, int num_sms);
 cudaError_t configure_kernels(const PassShape& ps);
@@ -45,11 +49,9 @@ void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s);
 void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s);
 void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s);
 
-// multi-GPU split tails: reduce per-block partials (1 block), and the
-// single-block finalisation after the host allreduce of red/redc.
+// multi-GPU: single-block finalisation after the NCCL allreduce of the
+// fixed-point cell sums (accg) and counts (cntg).
 enum Tail { TAIL_LOC = 0, TAIL_ASG = 1, TAIL_COST = 2, TAIL_REF = 3 };
-void launch_reduce(const RunParams& p, const PassShape& ps, int tail,
-                   cudaStream_t s);
 void launch_tail(const RunParams& p, int tail, cudaStream_t s);
 
 }  // namespace pc
