@@ -210,7 +210,7 @@ def run_gpu(args):
     common = dict(metric=metric, device=local, stream=stream.cuda_stream, world_size=world,
                   rank=rank, n_global=n if world > 1 else 0, row_offset=lo if world > 1 else 0,
                   nccl_unique_id=uid)
-    h = pk.Proclus(xdev, stats=True, **common)
+    h = pk.Proclus(xdev, stats=(world > 1), **common)
 
     def barrier():
         if world > 1:
@@ -227,6 +227,8 @@ def run_gpu(args):
     step_ms = []
     launches = 0
     iters = []
+    # timed region: the production path (single GPU: one CUDA graph per
+    # clustering whose while-node runs the iterative phase on the device)
     with ClockSampler(local) as clk:
         barrier()
         for s in range(args.steps):
@@ -240,8 +242,19 @@ def run_gpu(args):
             ev1.synchronize()
             step_ms.append(ev0.elapsed_time(ev1))
             iters.append(r.iterations)
-            st = h.stats()
-            launches += st["total_launches"]
+            launches += h.last_launches
+        barrier()
+    # per-kernel breakdown: the same steps again on an event-instrumented
+    # handle (every launch bracketed by CUDA events on the launching stream)
+    hs = pk.Proclus(xdev, stats=True, **dict(common, nccl_unique_id=None, world_size=1,
+                                             rank=0, n_global=0, row_offset=0)) \
+        if world == 1 else None
+    if hs is not None:
+        for s in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.zero_()
+            hs.run(k, l, seed=args.seed0 + s, labels=labels)
+            st = hs.stats()
             for kk, v in st["tail_ms"].items():
                 tails[kk] = tails.get(kk, 0.0) + v
             for kk, v in st["fallbacks"].items():
@@ -250,7 +263,11 @@ def run_gpu(args):
                 a = agg.setdefault(kind, dict(launches=0, ms=0.0, alg_bytes=0.0))
                 for f in ("launches", "ms", "alg_bytes"):
                     a[f] += st[kind][f]
-        barrier()
+        torch.cuda.synchronize()
+        hs.close()
+    else:
+        for kind in pk.STAT_KINDS:
+            agg.setdefault(kind, dict(launches=0, ms=0.0, alg_bytes=0.0))
     total_ms = sum(step_ms)
     if world > 1:
         t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
@@ -275,7 +292,10 @@ def run_gpu(args):
                 "traffic": ncu_traffic(dom), "peak_source": peak_src,
                 "bytes_per_launch": a["alg_bytes"] / max(a["launches"], 1),
                 "model": "data 4nd + Dist rows 4n per active slot (locality); data 4nd + u8 "
-                         "labels n (assign, cost)"}
+                         "labels n (assign, cost)",
+                "timing": "CUDA events around every launch on the launching stream, in an "
+                          "instrumented pass of the same steps/seeds right after the timed "
+                          "region (graph mode cannot bracket single kernels)"}
 
     # end to end through the public API with host buffers: H2D of the step's
     # data (pinned) + the whole run + D2H of labels / medoids / dims

@@ -592,7 +592,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
                                   uint64_t seed, proclus_result* out) {
   const int d = h->d;
   const int nM = (int)h->nM;
-  const PassShape ps = pass_shape(d, k, h->num_sms);
+  const PassShape ps = pass_shape(d, k, nM, h->num_sms);
   CK(configure_kernels(ps));
   CK(h->lab.ensure((size_t)2 * h->n_pad));
   CK(h->med.ensure((size_t)KMAX * d));
@@ -677,6 +677,9 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.st = h->st.p;
   p.P = ps.P;
   p.stages = ps.stages;
+  for (int q = 0; q < 4; ++q) p.lay[q] = ps.lay[q];
+  p.tl = ps.tl;
+  p.tail_smem = ps.tail_smem;
   p.nchunks = (h->n + ps.P - 1) / ps.P;
   p.fuse_tail = h->world == 1 ? 1 : 0;
   p.out_labels = h->out_labels.p;

@@ -61,6 +61,22 @@ struct TraceBufs {
   double* X;
 };
 
+// Byte offsets into a pass kernel's dynamic shared memory, computed on the
+// host (fixed offsets: no pointer arithmetic re-done inside the hot loops).
+struct SmemLayout {
+  int full, empty, buf, lab;                    // TMA ring and its mbarriers
+  int med, act, row, scale, cells, bal, acc, cnt, ex;
+  int tab, dl, nD, off, rcp, ctr, Dl, thr;
+  int tail;      // start of the tail scratch (reuses the ring region)
+  int bytes;     // total dynamic shared memory of the kernel
+  int nw;        // consumer warps
+};
+// Offsets (relative to SmemLayout::tail) of the single-block tail's scratch.
+struct TailLayout {
+  int S, X, Z, med, dev, dm, pool, fnd, bytes;
+};
+enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3 };
+
 struct RunParams {
   long long n;        // rows on this device
   long long n_pad;    // padded row count of the SoA layout (multiple of PAD_ALIGN)
@@ -98,6 +114,9 @@ struct RunParams {
   TraceBufs tr;
   int* out_labels;         // final labels [n] int32 (refinement)
   double* Delta;           // [k] outlier radii
+  SmemLayout lay[4];       // per KernelKind
+  TailLayout tl;
+  int tail_smem;           // dynamic smem of the standalone tail kernels
 };
 
 // ---- exact fp64 arithmetic: explicit round-to-nearest intrinsics so that

@@ -440,21 +440,30 @@ __device__ void flush_warps(const RunParams& p, const long long* acc_s, int nw, 
   }
 }
 
-// Exact total of accumulator c over the NCOPY copies; zeroes them.
+// Exact total of accumulator c over the NCOPY copies; zeroes them.  All
+// loads are issued before any store (one memory round trip).
 __device__ __forceinline__ long long take_acc(const RunParams& p, int c) {
-  long long s = 0;
   const size_t stride = (size_t)p.k * p.d;
+  long long v[NCOPY];
+#pragma unroll
+  for (int q = 0; q < NCOPY; ++q) v[q] = __ldcg(p.accg + q * stride + c);
+  long long s = 0;
+#pragma unroll
   for (int q = 0; q < NCOPY; ++q) {
-    s += __ldcg(p.accg + q * stride + c);
-    p.accg[q * stride + c] = 0;
+    s += v[q];
+    __stcg(p.accg + q * stride + c, 0ll);
   }
   return s;
 }
 __device__ __forceinline__ long long take_cnt(const RunParams& p, int c) {
+  long long v[NCOPY];
+#pragma unroll
+  for (int q = 0; q < NCOPY; ++q) v[q] = __ldcg(p.cntg + q * KMAX + c);
   long long s = 0;
+#pragma unroll
   for (int q = 0; q < NCOPY; ++q) {
-    s += __ldcg(p.cntg + q * KMAX + c);
-    p.cntg[q * KMAX + c] = 0;
+    s += v[q];
+    __stcg(p.cntg + q * KMAX + c, 0ll);
   }
   return s;
 }
@@ -548,407 +557,6 @@ static void size_pipe(CarveSize& cs, int rows, int P, int stages, bool with_lab)
   if (with_lab) cs.add<unsigned char>((size_t)stages * P);
 }
 
-// ============================================================ FindDimensions
-// Y_i, sigma_i, Z_ij (P:97-99, Alg 4 l.6-13, readings R2, R3) and the
-// selection of Alg 4 l.15-16 (reading R10): per medoid the two smallest by
-// (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j), found with a
-// block-wide radix select on order-preserving keys.  Whole block; X, Z,
-// dmask, dlist in global memory; nD[k] gets |D_i|.
-__device__ void zscore_select(const double* X, int k, int d, int l, double* Z,
-                              unsigned char* dmask, int* dlist, int* nD) {
-  __shared__ double Ys[KMAX], Ss[KMAX];
-  __shared__ unsigned int hist[256];
-  __shared__ unsigned long long prefix_s;
-  __shared__ int need_s;
-  __shared__ int tcount[TPB_MAX];
-  const int tid = threadIdx.x, bd = blockDim.x;
-  const int kd = k * d;
-  if (tid < k) {
-    const double* x = X + (long long)tid * d;
-    double Y = 0.0, s2 = 0.0;
-    for (int j = 0; j < d; ++j) Y = dadd(Y, x[j]);
-    Y = ddiv(Y, (double)d);
-    for (int j = 0; j < d; ++j) {
-      double u = dsub(x[j], Y);
-      s2 = dadd(s2, dmul(u, u));
-    }
-    Ys[tid] = Y;
-    Ss[tid] = __dsqrt_rn(ddiv(s2, (double)(d - 1)));
-  }
-  __syncthreads();
-  for (int c = tid; c < kd; c += bd) {
-    const int i = c / d;
-    const double sg = Ss[i];
-    Z[c] = (sg == 0.0) ? 0.0 : ddiv(dsub(X[c], Ys[i]), sg);
-    dmask[c] = 0;
-  }
-  __syncthreads();
-  if (tid < k) {  // two smallest per row, ties -> smaller j
-    const double* z = Z + (long long)tid * d;
-    int j1 = 0;
-    for (int j = 1; j < d; ++j)
-      if (z[j] < z[j1]) j1 = j;
-    int j2 = (j1 == 0) ? 1 : 0;
-    for (int j = 0; j < d; ++j)
-      if (j != j1 && z[j] < z[j2]) j2 = j;
-    dmask[(long long)tid * d + j1] = 1;
-    dmask[(long long)tid * d + j2] = 1;
-  }
-  __syncthreads();
-  const int R = k * l - 2 * k;
-  if (R > 0) {
-    if (tid == 0) {
-      prefix_s = 0ull;
-      need_s = R;
-    }
-    unsigned long long hmask = 0ull;
-    for (int shift = 56; shift >= 0; shift -= 8) {
-      for (int b = tid; b < 256; b += bd) hist[b] = 0u;
-      __syncthreads();
-      const unsigned long long pre = prefix_s;
-      for (int c = tid; c < kd; c += bd) {
-        if (dmask[c]) continue;
-        const unsigned long long key = sortable_key(Z[c]);
-        if ((key & hmask) == pre) atomicAdd(&hist[(key >> shift) & 255ull], 1u);
-      }
-      __syncthreads();
-      if (tid < 32) {  // warp scan over 256 bins, 8 per lane
-        unsigned loc[8], tot = 0;
-#pragma unroll
-        for (int b = 0; b < 8; ++b) {
-          loc[b] = hist[tid * 8 + b];
-          tot += loc[b];
-        }
-        unsigned x = tot;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          unsigned y = __shfl_up_sync(0xffffffffu, x, o);
-          if (tid >= o) x += y;
-        }
-        const unsigned before = x - tot;
-        const int need = need_s;
-        const bool here = (int)before < need && need <= (int)x;
-        const unsigned who = __ballot_sync(0xffffffffu, here);
-        if (here && tid == __ffs(who) - 1) {
-          unsigned cum = before;
-          int b = 0;
-          for (; b < 8; ++b) {
-            if ((int)(cum + loc[b]) >= need) break;
-            cum += loc[b];
-          }
-          need_s = need - (int)cum;
-          prefix_s = pre | ((unsigned long long)(tid * 8 + b) << shift);
-        }
-      }
-      hmask |= 255ull << shift;
-      __syncthreads();
-    }
-    const unsigned long long K = prefix_s;
-    const int need = need_s;  // how many cells with key == K to take
-    const int per = (kd + bd - 1) / bd;
-    const int c0 = tid * per, c1 = min(kd, c0 + per);
-    int eq = 0;
-    for (int c = c0; c < c1; ++c)
-      if (!dmask[c] && sortable_key(Z[c]) == K) ++eq;
-    tcount[tid] = eq;
-    __syncthreads();
-    if (tid == 0) {
-      int s = 0;
-      for (int t = 0; t < bd; ++t) {
-        int v = tcount[t];
-        tcount[t] = s;
-        s += v;
-      }
-    }
-    __syncthreads();
-    int rank = tcount[tid];
-    // each thread reads and writes only its own contiguous cell range here
-    for (int c = c0; c < c1; ++c) {
-      if (dmask[c]) continue;
-      const unsigned long long key = sortable_key(Z[c]);
-      if (key < K || (key == K && rank++ < need)) dmask[c] = 1;
-    }
-  }
-  __syncthreads();
-  if (tid < k) {
-    int t = 0;
-    for (int j = 0; j < d; ++j)
-      if (dmask[(long long)tid * d + j]) dlist[(long long)tid * d + t++] = j;
-    nD[tid] = t;
-  }
-  __syncthreads();
-}
-
-// ============================================================ iteration prologue
-// Medoid rows of MCur (fp64), delta_i (Alg 3 l.4-7, reading R6), and the
-// active slots of GPU-FAST-PROCLUS: new medoids get their Dist row computed,
-// cached ones with a changed radius get the band of Theorem 3.1.
-__device__ void prepare_iteration(const RunParams& p) {
-  DevState* st = p.st;
-  const int k = p.k, d = p.d;
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
-    const int i = e / d, j = e - i * d;
-    p.med[e] = (double)p.mrows[(long long)st->mcur[i] * d + j];
-  }
-  __threadfence_block();
-  __syncthreads();
-  if (threadIdx.x < k) {
-    const int i = threadIdx.x;
-    double m = CUDART_INF;
-    for (int j = 0; j < k; ++j) {
-      if (j == i) continue;
-      double t = full_dist(p.med + (long long)i * d, 1, p.med + (long long)j * d, d, p.metric);
-      if (t < m) m = t;
-    }
-    st->delta[i] = m;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    int na = 0;
-    for (int i = 0; i < k; ++i) {
-      const int mp = st->mcur[i];
-      const double dl = st->delta[i];
-      ActSlot a;
-      a.slot = i;
-      a.mpos = mp;
-      a.compute = p.found[mp] ? 0 : 1;
-      a.lam = 1;
-      if (!p.used[mp]) {
-        a.lo = -CUDART_INF;
-        a.hi = dl;
-      } else if (dl > p.dprev[mp]) {
-        a.lo = p.dprev[mp];
-        a.hi = dl;
-      } else if (dl < p.dprev[mp]) {
-        a.lo = dl;
-        a.hi = p.dprev[mp];
-        a.lam = -1;
-      } else {
-        continue;  // delta unchanged: Delta L_i is empty (eq 3)
-      }
-      st->act[na++] = a;
-    }
-    st->n_act = na;
-  }
-  __syncthreads();
-}
-
-__global__ void k_prepare(RunParams p) { prepare_iteration(p); }
-
-void launch_prepare(const RunParams& p, cudaStream_t s) { k_prepare<<<1, 256, 0, s>>>(p); }
-
-// ============================================================ tails
-// Locality tail: H and |L| updates of Theorem 3.2 / eq 6 and P:203 (in fixed
-// point, so the incremental H is exact integer arithmetic), DistFound /
-// delta' bookkeeping, X = H / |L| (P:201) and FindDimensions.
-__device__ void tail_locality(const RunParams& p) {
-  DevState* st = p.st;
-  const int d = p.d, na = st->n_act;
-  if (threadIdx.x == 0 && na > 0)  // byte model: data once + one Dist row per slot
-    st->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
-  for (int c = threadIdx.x; c < na * d; c += blockDim.x) {
-    const int a = c / d, j = c - a * d;
-    const ActSlot A = st->act[a];
-    const long long v = take_acc(p, c);
-    p.Hq[(long long)A.mpos * d + j] += (A.lam > 0 ? v : -v);
-  }
-  __syncthreads();
-  if (threadIdx.x < na) {
-    const ActSlot A = st->act[threadIdx.x];
-    const long long v = take_cnt(p, threadIdx.x);
-    p.nL[A.mpos] += (A.lam > 0 ? v : -v);
-    p.dprev[A.mpos] = st->delta[A.slot];
-    p.used[A.mpos] = 1;
-    p.found[A.mpos] = 1;
-  }
-  __threadfence_block();
-  __syncthreads();
-  for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
-    const int i = c / d, j = c - i * d;
-    const int mp = st->mcur[i];
-    p.X[c] = ddiv(dmul((double)p.Hq[(long long)mp * d + j], p.iscale[j]), (double)p.nL[mp]);
-  }
-  __threadfence_block();
-  __syncthreads();
-  zscore_select(p.X, p.k, d, p.l, p.Z, p.dmask, p.dlist, st->nD);
-  const int it = st->iterations;
-  if (p.tr.cap > 0 && it < p.tr.cap) {
-    for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
-      if (p.tr.X) p.tr.X[(long long)it * p.k * d + c] = p.X[c];
-      if (p.tr.dims) p.tr.dims[(long long)it * p.k * d + c] = p.dmask[c];
-    }
-    if (threadIdx.x < p.k) {
-      const int i = threadIdx.x;
-      if (p.tr.mcur) p.tr.mcur[it * p.k + i] = st->mcur[i];
-      if (p.tr.delta) p.tr.delta[it * p.k + i] = st->delta[i];
-      if (p.tr.nL) p.tr.nL[it * p.k + i] = p.nL[st->mcur[i]];
-    }
-  }
-  __syncthreads();
-}
-
-// Assign tail: |C_i| and the centroid mu_ij = sum / |C_i| on j in D_i (P:105).
-__device__ void tail_assign(const RunParams& p) {
-  DevState* st = p.st;
-  const int d = p.d;
-  __shared__ long long sz_s[KMAX];
-  if (threadIdx.x < p.k) {
-    sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
-    st->sizes[threadIdx.x] = sz_s[threadIdx.x];
-  }
-  __syncthreads();
-  for (int c = threadIdx.x; c < p.k * d; c += blockDim.x) {
-    const int i = c / d, t = c - i * d;
-    const long long sz = sz_s[i];
-    const long long v = take_acc(p, c);
-    double m = 0.0;
-    if (t < st->nD[i] && sz > 0) m = ddiv(dmul((double)v, p.iscale[p.dlist[c]]), (double)sz);
-    p.mu[c] = m;
-  }
-  __syncthreads();
-}
-
-// Cost tail: eq 1-2 with the |Data| denominator (eq 8, reading R4), then
-// Alg 1 l.10-14: keep the best, ComputeBadMedoids (P:91, reading R11),
-// replace bad medoids from M \ MBest (reading R12), stop after itrPat
-// iterations without improvement, and prepare the next iteration.
-__device__ void tail_cost(const RunParams& p) {
-  DevState* st = p.st;
-  const int k = p.k, d = p.d;
-  __shared__ int done_s;
-  __shared__ unsigned bad_s;
-  __shared__ int np_s;
-  double* dev = p.Z;  // scratch [k][d]: sum_{p in C_i} |x_pj - mu_ij|
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d, t = c - i * d;
-    const long long v = take_acc(p, c);
-    dev[c] = (t < st->nD[i]) ? dmul((double)v, p.iscale[p.dlist[c]]) : 0.0;
-  }
-  __threadfence_block();
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double cost = 0.0;
-    for (int i = 0; i < k; ++i) {
-      const long long c = st->sizes[i];
-      if (c == 0) continue;
-      double w = 0.0;
-      const int nd = st->nD[i];
-      for (int t = 0; t < nd; ++t) w = dadd(w, ddiv(dev[i * d + t], (double)c));
-      w = ddiv(w, (double)nd);
-      cost = dadd(cost, dmul((double)c, w));
-    }
-    cost = ddiv(cost, (double)p.n_total);
-    st->cost = cost;
-    st->itr += 1;
-    const int it = st->iterations;
-    st->iterations = it + 1;
-    const int improved = cost < st->cost_best;
-    st->improved = improved;
-    if (improved) {
-      st->itr = 0;
-      st->cost_best = cost;
-      for (int i = 0; i < k; ++i) {
-        st->mbest[i] = st->mcur[i];
-        st->sizes_best[i] = st->sizes[i];
-      }
-      st->best_buf = st->cur_buf;
-      st->cur_buf ^= 1;
-    }
-    unsigned bad = 0u;
-    const double thr = dmul(ddiv((double)p.n_total, (double)k), p.minDev);
-    int smallest = 0;
-    for (int i = 0; i < k; ++i) {
-      if ((double)st->sizes_best[i] < thr) bad |= 1u << i;
-      if (st->sizes_best[i] < st->sizes_best[smallest]) smallest = i;
-    }
-    if (!bad) bad = 1u << smallest;
-    bad_s = bad;
-    if (p.tr.cap > 0 && it < p.tr.cap) {
-      if (p.tr.cost) p.tr.cost[it] = cost;
-      if (p.tr.improved) p.tr.improved[it] = (unsigned char)improved;
-      for (int i = 0; i < k; ++i) {
-        if (p.tr.sizes) p.tr.sizes[it * k + i] = st->sizes[i];
-        if (p.tr.bad) p.tr.bad[it * k + i] = (bad >> i) & 1u;
-      }
-    }
-    for (int i = 0; i < k; ++i) st->mcur[i] = st->mbest[i];
-  }
-  __threadfence_block();
-  __syncthreads();
-  // pool = ascending positions of M not in MBest (warp compaction)
-  if (threadIdx.x < 32) {
-    int base = 0;
-    for (int t0 = 0; t0 < p.nM; t0 += 32) {
-      const int t = t0 + threadIdx.x;
-      bool inb = t >= p.nM;
-      if (!inb)
-        for (int i = 0; i < k; ++i) inb |= (st->mbest[i] == t);
-      const unsigned b = __ballot_sync(0xffffffffu, !inb);
-      if (!inb) p.pool[base + __popc(b & ((1u << threadIdx.x) - 1u))] = t;
-      base += __popc(b);
-    }
-    if (threadIdx.x == 0) np_s = base;
-  }
-  __threadfence_block();
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    // replacement draws (stream IT): the r-th remaining pool entry, in order
-    const unsigned bad = bad_s;
-    int np = np_s;
-    unsigned long long rng = st->rng;
-    for (int i = 0; i < k; ++i) {
-      if (!((bad >> i) & 1u) || np == 0) continue;
-      const int r = (int)sm64_uniform(&rng, (unsigned long long)np);
-      st->mcur[i] = p.pool[r];
-      for (int t = r; t + 1 < np; ++t) p.pool[t] = p.pool[t + 1];
-      --np;
-    }
-    st->rng = rng;
-    st->done = (st->itr >= p.itrPat || st->iterations >= p.max_iter) ? 1 : 0;
-    done_s = st->done;
-    if (p.use_cond)
-      cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, st->done ? 0u : 1u);
-  }
-  __threadfence_block();
-  __syncthreads();
-  if (!done_s) prepare_iteration(p);
-}
-
-// Refinement tail (Alg 1 l.16-17): X over CBest (empty cluster -> 0 row,
-// reading R15), FindDimensions -> D*, and the outlier radii
-// Delta_i = min_{j != i} seg_{D*_i}(m_i, m_j) (P:93, reading R5).
-__device__ void tail_refine(const RunParams& p) {
-  DevState* st = p.st;
-  const int k = p.k, d = p.d;
-  __shared__ long long sz_s[KMAX];
-  if (threadIdx.x < k) sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
-  __syncthreads();
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d, j = c - i * d;
-    const long long sz = sz_s[i];
-    const long long v = take_acc(p, c);
-    p.X[c] = sz > 0 ? ddiv(dmul((double)v, p.iscale[j]), (double)sz) : 0.0;
-  }
-  __threadfence_block();
-  __syncthreads();
-  zscore_select(p.X, k, d, p.l, p.Z, p.dmask, p.dlist, st->nD);
-  if (threadIdx.x < k) {
-    const int i = threadIdx.x, nd = st->nD[i];
-    const int* dl = p.dlist + (long long)i * d;
-    double m = CUDART_INF;
-    for (int j = 0; j < k; ++j) {
-      if (j == i) continue;
-      double s = 0.0;
-      for (int t = 0; t < nd; ++t)
-        s = dadd(s, fabs(dsub(p.med[(long long)i * d + dl[t]], p.med[(long long)j * d + dl[t]])));
-      const double q = ddiv(s, (double)nd);
-      if (q < m) m = q;
-    }
-    p.Delta[i] = m;
-  }
-  __syncthreads();
-}
-
 // ============================================================ certified tests
 // The fp32 value f approximates the oracle's fp64 value v with
 // |f - v| <= G * v (G from the error analysis of the fp32 evaluation,
@@ -1023,11 +631,499 @@ __device__ __noinline__ int exact_argmin(const float* __restrict__ x, int P,
   return bi;
 }
 
+// ============================================================ tails
+// The single-block steps between passes run on a shared-memory copy of the
+// device state (DevState) and of every small array they touch; global memory
+// is read in parallel at the start and written in parallel at the end, so no
+// thread waits on a chain of dependent global loads.
+struct TailMem {
+  DevState* S;
+  double* X;      // [k*d]
+  double* Z;      // [k*d]
+  double* med;    // [k*d] medoid rows, fp64
+  double* dev;    // [k*d]
+  unsigned char* dm;  // [k*d]
+  int* pool;      // [nM]
+  double* fnd;    // [3*KMAX]: found / used / delta' of the current slots
+};
+
+__device__ __forceinline__ TailMem tail_mem(const RunParams& p, unsigned char* base) {
+  const TailLayout& t = p.tl;
+  TailMem T;
+  T.S = (DevState*)(base + t.S);
+  T.X = (double*)(base + t.X);
+  T.Z = (double*)(base + t.Z);
+  T.med = (double*)(base + t.med);
+  T.dev = (double*)(base + t.dev);
+  T.dm = base + t.dm;
+  T.pool = (int*)(base + t.pool);
+  T.fnd = (double*)(base + t.fnd);
+  return T;
+}
+
+__device__ void state_load(const RunParams& p, DevState* S) {
+  const unsigned* src = (const unsigned*)p.st;
+  unsigned* dst = (unsigned*)S;
+  for (int i = threadIdx.x; i < (int)(sizeof(DevState) / 4); i += blockDim.x) dst[i] = __ldcg(src + i);
+  __syncthreads();
+}
+__device__ void state_store(const RunParams& p, const DevState* S) {
+  __syncthreads();
+  const unsigned* src = (const unsigned*)S;
+  unsigned* dst = (unsigned*)p.st;
+  for (int i = threadIdx.x; i < (int)(sizeof(DevState) / 4); i += blockDim.x) dst[i] = src[i];
+}
+
+// ------------------------------------------------------------ FindDimensions
+// Y_i, sigma_i, Z_ij (P:97-99, Alg 4 l.6-13, readings R2, R3) and the
+// selection of Alg 4 l.15-16 (reading R10): per medoid the two smallest by
+// (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j), found with a
+// block-wide radix select on order-preserving keys.  All in shared memory;
+// writes D as a mask (T.dm), |D_i| (S->nD) and, in global memory, the mask
+// and the ascending dimension lists used by the passes.
+__device__ void zscore_select_s(const RunParams& p, TailMem& T) {
+  __shared__ double Ys[KMAX], Ss[KMAX];
+  __shared__ unsigned int hist[256];
+  __shared__ unsigned long long prefix_s;
+  __shared__ int need_s;
+  __shared__ int tcount[TPB_MAX];
+  const int tid = threadIdx.x, bd = blockDim.x;
+  const int k = p.k, d = p.d, l = p.l, kd = k * d;
+  const double* X = T.X;
+  double* Z = T.Z;
+  unsigned char* dm = T.dm;
+  if (tid < k) {
+    const double* x = X + tid * d;
+    double Y = 0.0, s2 = 0.0;
+    for (int j = 0; j < d; ++j) Y = dadd(Y, x[j]);
+    Y = ddiv(Y, (double)d);
+    for (int j = 0; j < d; ++j) {
+      const double u = dsub(x[j], Y);
+      s2 = dadd(s2, dmul(u, u));
+    }
+    Ys[tid] = Y;
+    Ss[tid] = __dsqrt_rn(ddiv(s2, (double)(d - 1)));
+  }
+  __syncthreads();
+  for (int c = tid; c < kd; c += bd) {
+    const int i = c / d;
+    const double sg = Ss[i];
+    Z[c] = (sg == 0.0) ? 0.0 : ddiv(dsub(X[c], Ys[i]), sg);
+    dm[c] = 0;
+  }
+  __syncthreads();
+  if (tid < k) {  // two smallest per row, ties -> smaller j
+    const double* z = Z + tid * d;
+    int j1 = 0;
+    for (int j = 1; j < d; ++j)
+      if (z[j] < z[j1]) j1 = j;
+    int j2 = (j1 == 0) ? 1 : 0;
+    for (int j = 0; j < d; ++j)
+      if (j != j1 && z[j] < z[j2]) j2 = j;
+    dm[tid * d + j1] = 1;
+    dm[tid * d + j2] = 1;
+  }
+  __syncthreads();
+  const int R = k * l - 2 * k;
+  if (R > 0) {
+    if (tid == 0) {
+      prefix_s = 0ull;
+      need_s = R;
+    }
+    unsigned long long hmask = 0ull;
+    for (int shift = 56; shift >= 0; shift -= 8) {
+      for (int b = tid; b < 256; b += bd) hist[b] = 0u;
+      __syncthreads();
+      const unsigned long long pre = prefix_s;
+      for (int c = tid; c < kd; c += bd) {
+        if (dm[c]) continue;
+        const unsigned long long key = sortable_key(Z[c]);
+        if ((key & hmask) == pre) atomicAdd(&hist[(key >> shift) & 255ull], 1u);
+      }
+      __syncthreads();
+      if (tid < 32) {  // warp scan over 256 bins, 8 per lane
+        unsigned loc[8], tot = 0;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+          loc[b] = hist[tid * 8 + b];
+          tot += loc[b];
+        }
+        unsigned x = tot;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const unsigned y = __shfl_up_sync(0xffffffffu, x, o);
+          if (tid >= o) x += y;
+        }
+        const unsigned before = x - tot;
+        const int need = need_s;
+        const bool here = (int)before < need && need <= (int)x;
+        const unsigned who = __ballot_sync(0xffffffffu, here);
+        if (here && tid == __ffs(who) - 1) {
+          unsigned cum = before;
+          int b = 0;
+          for (; b < 8; ++b) {
+            if ((int)(cum + loc[b]) >= need) break;
+            cum += loc[b];
+          }
+          need_s = need - (int)cum;
+          prefix_s = pre | ((unsigned long long)(tid * 8 + b) << shift);
+        }
+      }
+      hmask |= 255ull << shift;
+      __syncthreads();
+    }
+    const unsigned long long K = prefix_s;
+    const int need = need_s;  // how many cells with key == K to take, in (i, j) order
+    const int per = (kd + bd - 1) / bd;
+    const int c0 = tid * per, c1 = min(kd, c0 + per);
+    int eq = 0;
+    for (int c = c0; c < c1; ++c)
+      if (!dm[c] && sortable_key(Z[c]) == K) ++eq;
+    tcount[tid] = eq;
+    __syncthreads();
+    if (tid < 32) {  // exclusive scan of tcount[0..bd) by one warp
+      int run = 0;
+      for (int b0 = 0; b0 < bd; b0 += 32) {
+        const int v = (b0 + tid < bd) ? tcount[b0 + tid] : 0;
+        int x = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(0xffffffffu, x, o);
+          if (tid >= o) x += y;
+        }
+        if (b0 + tid < bd) tcount[b0 + tid] = run + x - v;
+        run += __shfl_sync(0xffffffffu, x, 31);
+      }
+    }
+    __syncthreads();
+    int rank = tcount[tid];
+    for (int c = c0; c < c1; ++c) {  // own contiguous range only
+      if (dm[c]) continue;
+      const unsigned long long key = sortable_key(Z[c]);
+      if (key < K || (key == K && rank++ < need)) dm[c] = 1;
+    }
+  }
+  __syncthreads();
+  if (tid < k) {  // |D_i| and the ascending lists (global, for the passes)
+    int t = 0;
+    for (int j = 0; j < d; ++j)
+      if (dm[tid * d + j]) p.dlist[tid * d + t++] = j;
+    T.S->nD[tid] = t;
+  }
+  for (int c = tid; c < kd; c += bd) p.dmask[c] = dm[c];
+  __syncthreads();
+}
+
+// ------------------------------------------------------------ iteration prologue
+// Medoid rows of MCur (fp64), delta_i (Alg 3 l.4-7, reading R6), and the
+// active slots of GPU-FAST-PROCLUS: new medoids get their Dist row computed,
+// cached ones with a changed radius get the band of Theorem 3.1.
+__device__ void prepare_s(const RunParams& p, TailMem& T) {
+  DevState* S = T.S;
+  const int k = p.k, d = p.d;
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, j = e - i * d;
+    T.med[e] = (double)p.mrows[(long long)S->mcur[i] * d + j];
+  }
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    const int mp = S->mcur[i];
+    T.fnd[i] = p.found[mp];
+    T.fnd[KMAX + i] = p.used[mp];
+    T.fnd[2 * KMAX + i] = p.dprev[mp];
+  }
+  __syncthreads();
+  if (threadIdx.x < k) {
+    const int i = threadIdx.x;
+    double m = CUDART_INF;
+    for (int j = 0; j < k; ++j) {
+      if (j == i) continue;
+      const double t = full_dist(T.med + i * d, 1, T.med + j * d, d, p.metric);
+      if (t < m) m = t;
+    }
+    S->delta[i] = m;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int na = 0;
+    for (int i = 0; i < k; ++i) {
+      const double dl = S->delta[i];
+      const double dp = T.fnd[2 * KMAX + i];
+      ActSlot a;
+      a.slot = i;
+      a.mpos = S->mcur[i];
+      a.compute = T.fnd[i] != 0.0 ? 0 : 1;
+      a.lam = 1;
+      if (T.fnd[KMAX + i] == 0.0) {
+        a.lo = -CUDART_INF;
+        a.hi = dl;
+      } else if (dl > dp) {
+        a.lo = dp;
+        a.hi = dl;
+      } else if (dl < dp) {
+        a.lo = dl;
+        a.hi = dp;
+        a.lam = -1;
+      } else {
+        continue;  // delta unchanged: Delta L_i is empty (eq 3)
+      }
+      S->act[na++] = a;
+    }
+    S->n_act = na;
+  }
+  __syncthreads();
+}
+
+__global__ void k_prepare(RunParams p) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  TailMem T = tail_mem(p, smraw);
+  state_load(p, T.S);
+  prepare_s(p, T);
+  state_store(p, T.S);
+}
+
+void launch_prepare(const RunParams& p, cudaStream_t s) {
+  k_prepare<<<1, 256, p.tail_smem, s>>>(p);
+}
+
+// ------------------------------------------------------------ per-pass tails
+// Locality tail: H and |L| updates of Theorem 3.2 / eq 6 and P:203 (in fixed
+// point, so the incremental H is exact integer arithmetic), DistFound /
+// delta' bookkeeping, X = H / |L| (P:201) and FindDimensions.
+__device__ void tail_locality(const RunParams& p, TailMem& T) {
+  DevState* S = T.S;
+  const int d = p.d, k = p.k, na = S->n_act;
+  if (threadIdx.x == 0 && na > 0)  // byte model: data once + one Dist row per slot
+    S->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
+  for (int c = threadIdx.x; c < na * d; c += blockDim.x) {
+    const int a = c / d, j = c - a * d;
+    const ActSlot& A = S->act[a];
+    const long long v = take_acc(p, c);
+    p.Hq[(long long)A.mpos * d + j] += (A.lam > 0 ? v : -v);
+  }
+  if (threadIdx.x < na) {
+    const ActSlot& A = S->act[threadIdx.x];
+    const long long v = take_cnt(p, threadIdx.x);
+    p.nL[A.mpos] += (A.lam > 0 ? v : -v);
+    p.dprev[A.mpos] = S->delta[A.slot];
+    p.used[A.mpos] = 1;
+    p.found[A.mpos] = 1;
+  }
+  __threadfence_block();
+  __syncthreads();
+  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+    const int i = c / d, j = c - i * d;
+    const int mp = S->mcur[i];
+    T.X[c] = ddiv(dmul((double)p.Hq[(long long)mp * d + j], p.iscale[j]), (double)p.nL[mp]);
+  }
+  __syncthreads();
+  zscore_select_s(p, T);
+  const int it = S->iterations;
+  if (p.tr.cap > 0 && it < p.tr.cap) {
+    for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+      if (p.tr.X) p.tr.X[(long long)it * k * d + c] = T.X[c];
+      if (p.tr.dims) p.tr.dims[(long long)it * k * d + c] = T.dm[c];
+    }
+    if (threadIdx.x < k) {
+      const int i = threadIdx.x;
+      if (p.tr.mcur) p.tr.mcur[it * k + i] = S->mcur[i];
+      if (p.tr.delta) p.tr.delta[it * k + i] = S->delta[i];
+      if (p.tr.nL) p.tr.nL[it * k + i] = p.nL[S->mcur[i]];
+    }
+  }
+}
+
+// Assign tail: |C_i| and the centroid mu_ij = sum / |C_i| on j in D_i (P:105).
+__device__ void tail_assign(const RunParams& p, TailMem& T) {
+  DevState* S = T.S;
+  const int d = p.d, k = p.k;
+  if (threadIdx.x < k) S->sizes[threadIdx.x] = take_cnt(p, threadIdx.x);
+  __syncthreads();
+  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+    const int i = c / d, t = c - i * d;
+    const long long sz = S->sizes[i];
+    const long long v = take_acc(p, c);
+    double m = 0.0;
+    if (t < S->nD[i] && sz > 0) m = ddiv(dmul((double)v, p.iscale[p.dlist[c]]), (double)sz);
+    p.mu[c] = m;
+  }
+}
+
+// Cost tail: eq 1-2 with the |Data| denominator (eq 8, reading R4), then
+// Alg 1 l.10-14: keep the best, ComputeBadMedoids (P:91, reading R11),
+// replace bad medoids from M \ MBest (reading R12), stop after itrPat
+// iterations without improvement, and prepare the next iteration.
+__device__ void tail_cost(const RunParams& p, TailMem& T) {
+  DevState* S = T.S;
+  const int k = p.k, d = p.d;
+  __shared__ unsigned bad_s;
+  __shared__ int np_s;
+  __shared__ double cw_s[KMAX];
+  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+    const int i = c / d, t = c - i * d;
+    const long long v = take_acc(p, c);
+    T.dev[c] = (t < S->nD[i]) ? dmul((double)v, p.iscale[p.dlist[c]]) : 0.0;
+  }
+  __syncthreads();
+  if (threadIdx.x < k) {  // |C_i| * w_i of eq 1, one cluster per thread
+    const int i = threadIdx.x;
+    const long long c = S->sizes[i];
+    double cw = 0.0;
+    if (c != 0) {
+      double w = 0.0;
+      const int nd = S->nD[i];
+      for (int t = 0; t < nd; ++t) w = dadd(w, ddiv(T.dev[i * d + t], (double)c));
+      w = ddiv(w, (double)nd);
+      cw = dmul((double)c, w);
+    }
+    cw_s[i] = cw;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double cost = 0.0;
+    for (int i = 0; i < k; ++i)  // eq 2 / eq 8, i ascending; empty clusters add 0
+      if (S->sizes[i] != 0) cost = dadd(cost, cw_s[i]);
+    cost = ddiv(cost, (double)p.n_total);
+    S->cost = cost;
+    S->itr += 1;
+    const int it = S->iterations;
+    S->iterations = it + 1;
+    const int improved = cost < S->cost_best;
+    S->improved = improved;
+    if (improved) {
+      S->itr = 0;
+      S->cost_best = cost;
+      for (int i = 0; i < k; ++i) {
+        S->mbest[i] = S->mcur[i];
+        S->sizes_best[i] = S->sizes[i];
+      }
+      S->best_buf = S->cur_buf;
+      S->cur_buf ^= 1;
+    }
+    unsigned bad = 0u;
+    const double thr = dmul(ddiv((double)p.n_total, (double)k), p.minDev);
+    int smallest = 0;
+    for (int i = 0; i < k; ++i) {
+      if ((double)S->sizes_best[i] < thr) bad |= 1u << i;
+      if (S->sizes_best[i] < S->sizes_best[smallest]) smallest = i;
+    }
+    if (!bad) bad = 1u << smallest;
+    bad_s = bad;
+    if (p.tr.cap > 0 && it < p.tr.cap) {
+      if (p.tr.cost) p.tr.cost[it] = cost;
+      if (p.tr.improved) p.tr.improved[it] = (unsigned char)improved;
+      for (int i = 0; i < k; ++i) {
+        if (p.tr.sizes) p.tr.sizes[it * k + i] = S->sizes[i];
+        if (p.tr.bad) p.tr.bad[it * k + i] = (bad >> i) & 1u;
+      }
+    }
+    for (int i = 0; i < k; ++i) S->mcur[i] = S->mbest[i];
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {  // pool = ascending positions of M not in MBest
+    int base = 0;
+    for (int t0 = 0; t0 < p.nM; t0 += 32) {
+      const int t = t0 + threadIdx.x;
+      bool inb = t >= p.nM;
+      if (!inb)
+        for (int i = 0; i < k; ++i) inb |= (S->mbest[i] == t);
+      const unsigned b = __ballot_sync(0xffffffffu, !inb);
+      if (!inb) T.pool[base + __popc(b & ((1u << threadIdx.x) - 1u))] = t;
+      base += __popc(b);
+    }
+    if (threadIdx.x == 0) np_s = base;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    // replacement draws (stream IT): the r-th remaining pool entry, in order
+    const unsigned bad = bad_s;
+    int np = np_s;
+    unsigned long long rng = S->rng;
+    for (int i = 0; i < k; ++i) {
+      if (!((bad >> i) & 1u) || np == 0) continue;
+      const int r = (int)sm64_uniform(&rng, (unsigned long long)np);
+      S->mcur[i] = T.pool[r];
+      for (int t = r; t + 1 < np; ++t) T.pool[t] = T.pool[t + 1];
+      --np;
+    }
+    S->rng = rng;
+    S->done = (S->itr >= p.itrPat || S->iterations >= p.max_iter) ? 1 : 0;
+    if (p.use_cond)
+      cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, S->done ? 0u : 1u);
+  }
+  __syncthreads();
+  if (!S->done) prepare_s(p, T);
+}
+
+// Refinement tail (Alg 1 l.16-17): X over CBest (empty cluster -> 0 row,
+// reading R15), FindDimensions -> D*, and the outlier radii
+// Delta_i = min_{j != i} seg_{D*_i}(m_i, m_j) (P:93, reading R5).
+__device__ void tail_refine(const RunParams& p, TailMem& T) {
+  DevState* S = T.S;
+  const int k = p.k, d = p.d;
+  __shared__ long long sz_s[KMAX];
+  if (threadIdx.x < k) sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, j = e - i * d;
+    T.med[e] = (double)p.mrows[(long long)S->mbest[i] * d + j];
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+    const int i = c / d, j = c - i * d;
+    const long long sz = sz_s[i];
+    const long long v = take_acc(p, c);
+    T.X[c] = sz > 0 ? ddiv(dmul((double)v, p.iscale[j]), (double)sz) : 0.0;
+  }
+  __syncthreads();
+  zscore_select_s(p, T);
+  if (threadIdx.x < k) {
+    const int i = threadIdx.x;
+    double m = CUDART_INF;
+    for (int j = 0; j < k; ++j) {
+      if (j == i) continue;
+      double s = 0.0;
+      int nd = 0;
+      for (int t = 0; t < d; ++t) {
+        if (!T.dm[i * d + t]) continue;
+        s = dadd(s, fabs(dsub(T.med[i * d + t], T.med[j * d + t])));
+        ++nd;
+      }
+      const double q = ddiv(s, (double)nd);
+      if (q < m) m = q;
+    }
+    p.Delta[i] = m;
+  }
+}
+
+// Run a tail: load the state into shared memory, run it, store it back.
+#define RUN_TAIL(FN, KIND)                                          \
+  do {                                                              \
+    const unsigned long long t0_ = gtimer();                        \
+    TailMem T_ = tail_mem(p, smraw + p.lay[LAYK].tail);             \
+    state_load(p, T_.S);                                            \
+    FN(p, T_);                                                      \
+    __syncthreads();                                                \
+    if (threadIdx.x == 0) T_.S->tail_ns[KIND] += gtimer() - t0_;    \
+    state_store(p, T_.S);                                           \
+  } while (0)
+
 // ============================================================ pass kernels
 // Block = NW consumer warps + 1 producer warp.  Consumer warp w owns the
 // sub-chunk of 32*PPT points starting at q0 = w*32*PPT of every chunk.
+// Shared-memory arrays live at host-computed offsets (p.lay[kind]).
+#define SMP(T, field) reinterpret_cast<T*>(smraw + L.field)
+
 __device__ __forceinline__ long long chunks_of_block(const RunParams& p) {
   return (p.nchunks > blockIdx.x) ? (p.nchunks - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+}
+
+__device__ __forceinline__ Pipe pipe_of(const SmemLayout& L, unsigned char* smraw, int rows) {
+  Pipe R;
+  R.full = SMP(unsigned long long, full);
+  R.empty = SMP(unsigned long long, empty);
+  R.buf = SMP(float, buf);
+  R.lab = L.lab >= 0 ? SMP(unsigned char, lab) : nullptr;
+  R.rows = rows;
+  return R;
 }
 
 // Cells (i, t < |D_i|) in cluster order: exclusive scan of |D_i| by warp 0,
@@ -1049,40 +1145,67 @@ __device__ int build_cells(Cell* cells, const int* nD_s, int k, int d, int* off_
   __syncthreads();
   for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
     const int i = e / d, t = e - i * d;
-    if (t < nD_s[i])
-      cells[off_s[i] + t] = Cell{i, dl_s[e], e, ctr_s ? ctr_s[e] : 0.0};
+    if (t < nD_s[i]) cells[off_s[i] + t] = Cell{i, dl_s[e], e, ctr_s ? ctr_s[e] : 0.0};
   }
   __syncthreads();
   return off_s[KMAX];
 }
 
+// fp32 certified thresholds of one band (lo, hi]: a fp32 value f with
+// |f - v| <= G v decides v <= T when f < T(1-G) (then "<=") or f > T(1+G)
+// (then ">"); the bounds are rounded outwards to fp32 once per launch.
+struct Thr {
+  float in_hi, out_hi;  // f < in_hi: v <= hi;  f > out_hi: v > hi
+  float in_lo, out_lo;  // f > out_lo: v > lo;  f < in_lo: v <= lo
+};
+__device__ __forceinline__ Thr make_thr(double lo, double hi, double G) {
+  Thr t;
+  const bool hok = hi >= 1e-30 && hi < 1e30;
+  t.in_hi = hok ? __double2float_rd(hi * (1.0 - G)) : -1.0f;
+  t.out_hi = hok ? __double2float_ru(hi * (1.0 + G)) : CUDART_INF_F;
+  if (lo == -CUDART_INF) {
+    t.out_lo = -1.0f;  // every f >= 0 is above
+    t.in_lo = -2.0f;
+  } else {
+    const bool lok = lo >= 1e-30 && lo < 1e30;
+    t.in_lo = lok ? __double2float_rd(lo * (1.0 - G)) : -1.0f;
+    t.out_lo = lok ? __double2float_ru(lo * (1.0 + G)) : CUDART_INF_F;
+  }
+  return t;
+}
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
 // One point per lane; the cached Dist rows of the active slots arrive through
-// the same TMA ring as the data (rows d..).
-template <bool XREG>
+// the same TMA ring as the data (rows d..).  DR: coordinates in registers.
+template <int DR>
 __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_LOC];
+#define LAYK KK_LOC
   const int P = p.P, d = p.d, k = p.k;
-  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int na = st->n_act;
   const int ncap = k * d;
-  Carve cv(smraw);
-  Pipe R = carve_pipe(cv, p, d + k, false);
-  float* med_s = cv.take<float>((size_t)k * d);
-  ActSlot* act_s = cv.take<ActSlot>(KMAX);
-  int* row_s = cv.take<int>(KMAX);
-  double* scale_s = cv.take<double>(d);
-  Cell* cells = cv.take<Cell>((size_t)ncap);
-  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX);
-  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
-  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
-  ExtraRows* ex = cv.take<ExtraRows>(1);
+  const Pipe R = pipe_of(L, smraw, d + k);
+  float* med_s = SMP(float, med);
+  ActSlot* act_s = SMP(ActSlot, act);
+  int* row_s = SMP(int, row);
+  double* scale_s = SMP(double, scale);
+  Cell* cells = SMP(Cell, cells);
+  unsigned* bal_s = SMP(unsigned, bal);
+  long long* acc_s = SMP(long long, acc);
+  long long* cnt_s = SMP(long long, cnt);
+  ExtraRows* ex = SMP(ExtraRows, ex);
+  Thr* thr_s = SMP(Thr, thr);
   const long long nmy = chunks_of_block(p);
   const double G = (double)(d + 8) * 5.9604644775390625e-08;  // (d+8) 2^-24
 
-  for (int a = threadIdx.x; a < na; a += blockDim.x) act_s[a] = st->act[a];
+  for (int a = threadIdx.x; a < na; a += blockDim.x) {
+    act_s[a] = st->act[a];
+    thr_s[a] = make_thr(st->act[a].lo, st->act[a].hi, G);
+  }
   for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
   for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
   for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
@@ -1093,15 +1216,18 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
     const bool cached = a < na && !act_s[a].compute;
     const unsigned b = __ballot_sync(0xffffffffu, cached);
     const int r = __popc(b & ((1u << a) - 1u));
-    if (a < na) row_s[a] = cached ? d + r : -1;
+    if (a < na) row_s[a] = cached ? (d + r) * P : -1;
     if (cached) ex->src[r] = p.dist + (size_t)act_s[a].mpos * p.n_pad;
     if (a == 0) ex->n = __popc(b);
   }
-  for (int e = threadIdx.x; e < na * d; e += blockDim.x) {
-    const int a = e / d, j = e - a * d;
-    const float m = p.mrows[(long long)act_s[a].mpos * d + j];
+  // medoid rows at stride MS (zero padded to DR for float4 loads)
+  constexpr int MSD = DR > 0 ? DR : 0;
+  const int MS = MSD > 0 ? MSD : d;
+  for (int e = threadIdx.x; e < na * MS; e += blockDim.x) {
+    const int a = e / MS, j = e - a * MS;
+    const float m = j < d ? p.mrows[(long long)act_s[a].mpos * d + j] : 0.f;
     med_s[e] = m;
-    cells[e] = Cell{a, j, e, (double)m};
+    if (j < d) cells[a * d + j] = Cell{a, j, a * d + j, (double)m};
   }
   __syncthreads();
   long long nfb = 0;
@@ -1112,35 +1238,66 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
       unsigned* bal = bal_s + w * KMAX;
       long long* acc = acc_s + (size_t)w * ncap;
       const int q = w * 32 + lane;
-      for (long long i = 0; i < nmy; ++i) {
+      const int metric = p.metric;
+      long long gp = (long long)blockIdx.x * P + q;
+      const long long gstep = (long long)gridDim.x * P;
+      for (long long i = 0; i < nmy; ++i, gp += gstep) {
         const int stg = (int)(i % p.stages);
-        const long long gp = (blockIdx.x + i * gridDim.x) * (long long)P + q;
         mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
         const float* xs = R.buf + (size_t)stg * R.rows * P;
         const bool valid = gp < p.n;
-        float xr[DREG];
-        if (XREG) {
+        float xr[DR > 0 ? DR : 1];
+        if (DR > 0) {
 #pragma unroll
-          for (int j = 0; j < DREG; ++j) xr[j] = (j < d) ? xs[j * P + q] : 0.f;
+          for (int j = 0; j < DR; ++j) xr[j] = (j < d) ? xs[j * P + q] : 0.f;
         }
         for (int a = 0; a < na; ++a) {
-          const ActSlot A = act_s[a];
+          const int rs = row_s[a];
           bool in = false;
           if (valid) {
             float f;
-            if (A.compute) {  // compute distances only once
-              f = XREG ? approx_full_reg(xr, med_s + a * d, d, p.metric)
-                       : approx_full(xs + q, P, med_s + a * d, d, p.metric);
-              p.dist[(long long)A.mpos * p.n_pad + gp] = f;
+            if (rs < 0) {  // compute distances only once
+              const float* m = med_s + a * MS;
+              float s = 0.f;
+              if (DR > 0) {  // padded coordinates are 0 on both sides
+                const float4* m4 = reinterpret_cast<const float4*>(m);
+                if (metric == 1) {
+#pragma unroll
+                  for (int j4 = 0; j4 < MSD / 4; ++j4) {
+                    const float4 v = m4[j4];
+                    s += fabsf(xr[4 * j4] - v.x) + fabsf(xr[4 * j4 + 1] - v.y) +
+                         fabsf(xr[4 * j4 + 2] - v.z) + fabsf(xr[4 * j4 + 3] - v.w);
+                  }
+                } else {
+                  float s1 = 0.f;
+#pragma unroll
+                  for (int j4 = 0; j4 < MSD / 4; ++j4) {
+                    const float4 v = m4[j4];
+                    const float t0 = xr[4 * j4] - v.x, t1 = xr[4 * j4 + 1] - v.y;
+                    const float t2 = xr[4 * j4 + 2] - v.z, t3 = xr[4 * j4 + 3] - v.w;
+                    s = fmaf(t0, t0, s);
+                    s1 = fmaf(t1, t1, s1);
+                    s = fmaf(t2, t2, s);
+                    s1 = fmaf(t3, t3, s1);
+                  }
+                  s = sqrtf(s + s1);
+                }
+              } else {
+                s = approx_full(xs + q, P, m, d, metric);
+              }
+              f = s;
+              p.dist[(long long)act_s[a].mpos * p.n_pad + gp] = f;
             } else {
-              f = xs[row_s[a] * P + q];
+              f = xs[rs + q];
             }
-            const int rhi = cert_le(f, A.hi, G);
-            const int rlo = (A.lo == -CUDART_INF) ? 0 : cert_le(f, A.lo, G);
-            if (rhi >= 0 && rlo >= 0) {
-              in = (rhi == 1) && (rlo == 0);  // v <= hi and not v <= lo
-            } else {
-              const double dv = full_dist(xs + q, P, med_s + a * d, d, p.metric);
+            const Thr t = thr_s[a];
+            if (f < t.in_hi && f > t.out_lo) {
+              in = true;
+            } else if (f > t.out_hi || f < t.in_lo) {
+              in = false;
+            } else {  // within the fp32 error bound: the oracle's fp64 value
+              const ActSlot A = act_s[a];
+              const double dv = full_dist(xs + q, P, med_s + a * MS, d, metric);
               in = (dv > A.lo) && (dv <= A.hi);
               ++nfb;
             }
@@ -1160,39 +1317,40 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   if (nfb) atomicAdd((unsigned long long*)&st->fallback[0], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[0])) return;
-  const unsigned long long t0 = gtimer();
-  tail_locality(p);
-  if (threadIdx.x == 0) st->tail_ns[0] += gtimer() - t0;
+  RUN_TAIL(tail_locality, 0);
+#undef LAYK
 }
 
 // --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8).
 // PPT points per lane so every term-table entry loaded serves PPT points.
-struct Term {
-  int joff;  // j * P
+struct __align__(8) Term {
+  int joff;  // byte offset of row j in a ring stage: j * P * 4
   float m;   // m_ij
 };
+#define LDX(base, boff) (*reinterpret_cast<const float*>(reinterpret_cast<const char*>(base) + (boff)))
 
 template <int PPT>
 __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_ASG];
+#define LAYK KK_ASG
   const int P = p.P, d = p.d, k = p.k;
-  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ncap = k * d;
-  Carve cv(smraw);
-  Pipe R = carve_pipe(cv, p, d, false);
-  float* med_s = cv.take<float>((size_t)k * d);
-  Term* tab_s = cv.take<Term>((size_t)k * d);
-  int* dl_s = cv.take<int>((size_t)k * d);
-  int* nD_s = cv.take<int>(KMAX);
-  int* off_s = cv.take<int>(KMAX + 1);
-  float* rcp_s = cv.take<float>(KMAX);
-  double* scale_s = cv.take<double>(d);
-  Cell* cells = cv.take<Cell>((size_t)ncap);
-  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX * PPT);
-  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
-  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
+  const Pipe R = pipe_of(L, smraw, d);
+  float* med_s = SMP(float, med);
+  Term* tab_s = SMP(Term, tab);
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nD);
+  int* off_s = SMP(int, off);
+  float* rcp_s = SMP(float, rcp);
+  double* scale_s = SMP(double, scale);
+  Cell* cells = SMP(Cell, cells);
+  unsigned* bal_s = SMP(unsigned, bal);
+  long long* acc_s = SMP(long long, acc);
+  long long* cnt_s = SMP(long long, cnt);
   unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
   const long long nmy = chunks_of_block(p);
 
@@ -1214,7 +1372,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     const int i = e / d, t = e - i * d;
     if (t < nD_s[i]) {
       const int j = dl_s[e];
-      tab_s[e].joff = j * P;
+      tab_s[e].joff = j * P * 4;
       tab_s[e].m = med_s[i * d + j];
     }
   }
@@ -1229,9 +1387,10 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     unsigned* bal = bal_s + w * KMAX * PPT;
     long long* acc = acc_s + (size_t)w * ncap;
     const int q0 = w * 32 * PPT;
-    for (long long i = 0; i < nmy; ++i) {
+    long long base = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    for (long long i = 0; i < nmy; ++i, base += gstep) {
       const int stg = (int)(i % p.stages);
-      const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
       mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const float* xq = xs + q0 + lane;
@@ -1243,9 +1402,9 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         second[u] = CUDART_INF_F;
         bi[u] = 0;
       }
-      for (int c = 0; c < k; ++c) {
+      const Term* tb = tab_s;
+      for (int c = 0; c < k; ++c, tb += d) {
         const int nd = nD_s[c];
-        const Term* tb = tab_s + c * d;
         // fp32 partial sums in any order: the certified bound only needs the
         // number of terms; 4 terms in flight per point
         float s[PPT], s2[PPT];
@@ -1260,28 +1419,32 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
 #pragma unroll
           for (int u = 0; u < PPT; ++u) {
             const float* xu = xq + u * 32;
-            const float a0 = fabsf(xu[e0.joff] - e0.m), a1 = fabsf(xu[e1.joff] - e1.m);
-            const float a2 = fabsf(xu[e2.joff] - e2.m), a3 = fabsf(xu[e3.joff] - e3.m);
-            s[u] += a0 + a1;
-            s2[u] += a2 + a3;
+            s[u] += fabsf(LDX(xu, e0.joff) - e0.m) + fabsf(LDX(xu, e1.joff) - e1.m);
+            s2[u] += fabsf(LDX(xu, e2.joff) - e2.m) + fabsf(LDX(xu, e3.joff) - e3.m);
           }
         }
-        for (; t < nd; ++t) {
+        if (t + 2 <= nd) {
+          const Term e0 = tb[t], e1 = tb[t + 1];
+#pragma unroll
+          for (int u = 0; u < PPT; ++u) {
+            const float* xu = xq + u * 32;
+            s[u] += fabsf(LDX(xu, e0.joff) - e0.m);
+            s2[u] += fabsf(LDX(xu, e1.joff) - e1.m);
+          }
+          t += 2;
+        }
+        if (t < nd) {
           const Term e = tb[t];
 #pragma unroll
-          for (int u = 0; u < PPT; ++u) s[u] += fabsf(xq[u * 32 + e.joff] - e.m);
+          for (int u = 0; u < PPT; ++u) s[u] += fabsf(LDX(xq + u * 32, e.joff) - e.m);
         }
         const float r = rcp_s[c];
 #pragma unroll
         for (int u = 0; u < PPT; ++u) {
           const float qv = (s[u] + s2[u]) * r;
-          if (qv < best[u]) {
-            second[u] = best[u];
-            best[u] = qv;
-            bi[u] = c;
-          } else if (qv < second[u]) {
-            second[u] = qv;
-          }
+          second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);
+          bi[u] = qv < best[u] ? c : bi[u];
+          best[u] = fminf(best[u], qv);
         }
       }
       int lbl[PPT];
@@ -1291,9 +1454,8 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         const long long gp = base + q;
         lbl[u] = -1;
         if (gp >= p.n) continue;
-        const double b = (double)best[u], s2v = (double)second[u];
-        const bool certain =
-            (b >= 1e-30) && (s2v < 1e30) && (s2v * (1.0 - G) > b * (1.0 + G));
+        const bool certain = (best[u] >= 1e-30f) && (second[u] < 1e30f) &&
+                             ((double)second[u] * (1.0 - G) > (double)best[u] * (1.0 + G));
         lbl[u] = bi[u];
         if (!certain) {
           lbl[u] = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
@@ -1301,16 +1463,27 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         }
         lab[gp] = (unsigned char)lbl[u];
       }
-      for (int c = 0; c < k; ++c)
+      {  // one ballot per (cluster, u): lane c keeps cluster c's masks
+        unsigned mine[PPT];
 #pragma unroll
-        for (int u = 0; u < PPT; ++u) put_ballot(bal, c * PPT + u, lbl[u] == c);
-      __syncwarp();
-      if (lane < k) {
-        int cn = 0;
+        for (int u = 0; u < PPT; ++u) mine[u] = 0u;
+        for (int c = 0; c < k; ++c)
 #pragma unroll
-        for (int u = 0; u < PPT; ++u) cn += __popc(bal[lane * PPT + u]);
-        cnt_s[w * KMAX + lane] += cn;
+          for (int u = 0; u < PPT; ++u) {
+            const unsigned b = __ballot_sync(0xffffffffu, lbl[u] == c);
+            if (lane == c) mine[u] = b;
+          }
+        if (lane < k) {
+          int cn = 0;
+#pragma unroll
+          for (int u = 0; u < PPT; ++u) {
+            bal[lane * PPT + u] = mine[u];
+            cn += __popc(mine[u]);
+          }
+          cnt_s[w * KMAX + lane] += cn;
+        }
       }
+      __syncwarp();
       warp_cells<0, PPT>(xs, P, q0, cells, ncell, bal, acc, scale_s);
       pipe_release(R, stg);
     }
@@ -1320,9 +1493,8 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[1])) return;
-  const unsigned long long t0 = gtimer();
-  tail_assign(p);
-  if (threadIdx.x == 0) st->tail_ns[1] += gtimer() - t0;
+  RUN_TAIL(tail_assign, 1);
+#undef LAYK
 }
 
 // --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) + control tail, and the
@@ -1334,20 +1506,21 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
   DevState* st = p.st;
   if (!REF && st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_LSUM];
+#define LAYK KK_LSUM
   const int P = p.P, d = p.d, k = p.k;
-  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ncap = k * d;
-  Carve cv(smraw);
-  Pipe R = carve_pipe(cv, p, d, true);
-  double* ctr_s = cv.take<double>((size_t)k * d);
-  int* dl_s = cv.take<int>((size_t)k * d);
-  int* nD_s = cv.take<int>(KMAX);
-  int* off_s = cv.take<int>(KMAX + 1);
-  double* scale_s = cv.take<double>(d);
-  Cell* cells = cv.take<Cell>((size_t)ncap);
-  unsigned* bal_s = cv.take<unsigned>((size_t)nw * KMAX);
-  long long* acc_s = cv.take<long long>((size_t)nw * ncap);
-  long long* cnt_s = cv.take<long long>((size_t)nw * KMAX);
+  const Pipe R = pipe_of(L, smraw, d);
+  double* ctr_s = SMP(double, ctr);
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nD);
+  int* off_s = SMP(int, off);
+  double* scale_s = SMP(double, scale);
+  Cell* cells = SMP(Cell, cells);
+  unsigned* bal_s = SMP(unsigned, bal);
+  long long* acc_s = SMP(long long, acc);
+  long long* cnt_s = SMP(long long, cnt);
   const unsigned char* lab =
       REF ? (st->best_buf ? p.lab1 : p.lab0) : (st->cur_buf ? p.lab1 : p.lab0);
   const long long nmy = chunks_of_block(p);
@@ -1369,15 +1542,24 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
     unsigned* bal = bal_s + w * KMAX;
     long long* acc = acc_s + (size_t)w * ncap;
     const int q = w * 32 + lane;
-    for (long long i = 0; i < nmy; ++i) {
+    long long gp = (long long)blockIdx.x * P + q;
+    const long long gstep = (long long)gridDim.x * P;
+    for (long long i = 0; i < nmy; ++i, gp += gstep) {
       const int stg = (int)(i % p.stages);
-      const long long gp = (blockIdx.x + i * gridDim.x) * (long long)P + q;
       mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const int lb = gp < p.n ? (int)R.lab[(size_t)stg * P + q] : -1;
-      for (int c = 0; c < k; ++c) put_ballot(bal, c, lb == c);
+      // one ballot per cluster: lane c of the warp keeps cluster c's mask
+      unsigned mine = 0u;
+      for (int c = 0; c < k; ++c) {
+        const unsigned b = __ballot_sync(0xffffffffu, lb == c);
+        if (lane == c) mine = b;
+      }
+      if (lane < k) {
+        bal[lane] = mine;
+        if (REF) cnt_s[w * KMAX + lane] += __popc(mine);
+      }
       __syncwarp();
-      if (REF && lane < k) cnt_s[w * KMAX + lane] += __popc(bal[lane]);
       warp_cells<1, 1>(xs, P, w * 32, cells, ncell, bal, acc, scale_s);
       pipe_release(R, stg);
     }
@@ -1386,16 +1568,11 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
   flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, REF ? k : 0);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[REF ? 3 : 2])) return;
-  const unsigned long long t0 = gtimer();
-  if (REF) {
-    for (int e = threadIdx.x; e < k * d; e += blockDim.x) p.med[e] = ctr_s[e];
-    __threadfence_block();
-    __syncthreads();
-    tail_refine(p);
-  } else {
-    tail_cost(p);
-  }
-  if (threadIdx.x == 0) st->tail_ns[REF ? 3 : 2] += gtimer() - t0;
+  if (REF)
+    RUN_TAIL(tail_refine, 3);
+  else
+    RUN_TAIL(tail_cost, 2);
+#undef LAYK
 }
 
 // --- Final AssignPoints with D* (Alg 1 l.18) and RemoveOutliers (l.19):
@@ -1404,16 +1581,16 @@ template <int PPT>
 __global__ void __launch_bounds__(160) k_final(RunParams p) {
   DevState* st = p.st;
   extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_FIN];
   const int P = p.P, d = p.d, k = p.k;
-  const int nw = blockDim.x / 32 - 1, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  Carve cv(smraw);
-  Pipe R = carve_pipe(cv, p, d, false);
-  float* med_s = cv.take<float>((size_t)k * d);
-  Term* tab_s = cv.take<Term>((size_t)k * d);
-  int* dl_s = cv.take<int>((size_t)k * d);
-  int* nD_s = cv.take<int>(KMAX);
-  float* rcp_s = cv.take<float>(KMAX);
-  double* Dl_s = cv.take<double>(KMAX);
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const Pipe R = pipe_of(L, smraw, d);
+  float* med_s = SMP(float, med);
+  Term* tab_s = SMP(Term, tab);
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nD);
+  float* rcp_s = SMP(float, rcp);
+  double* Dl_s = SMP(double, Dl);
   const long long nmy = chunks_of_block(p);
   for (int i = threadIdx.x; i < k; i += blockDim.x) {
     nD_s[i] = st->nD[i];
@@ -1431,7 +1608,7 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
     const int i = e / d, t = e - i * d;
     if (t < nD_s[i]) {
       const int j = dl_s[e];
-      tab_s[e].joff = j * P;
+      tab_s[e].joff = j * P * 4;
       tab_s[e].m = med_s[i * d + j];
     }
   }
@@ -1464,10 +1641,10 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
           float s = 0.f, s2 = 0.f;
           int t = 0;
           for (; t + 2 <= nd; t += 2) {
-            s += fabsf(xs[tb[t].joff + q] - tb[t].m);
-            s2 += fabsf(xs[tb[t + 1].joff + q] - tb[t + 1].m);
+            s += fabsf(LDX(xs + q, tb[t].joff) - tb[t].m);
+            s2 += fabsf(LDX(xs + q, tb[t + 1].joff) - tb[t + 1].m);
           }
-          if (t < nd) s += fabsf(xs[tb[t].joff + q] - tb[t].m);
+          if (t < nd) s += fabsf(LDX(xs + q, tb[t].joff) - tb[t].m);
           const float qv = (s + s2) * rcp_s[c];
           if (qv < best) {
             second = best;
@@ -1500,67 +1677,71 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
 
 // ============================================================ multi-GPU tail
 __global__ void k_tail(RunParams p, int tail) {
+  extern __shared__ __align__(16) unsigned char smraw[];
   DevState* st = p.st;
-  if (tail == TAIL_LOC) {
-    if (st->done) return;
-    tail_locality(p);
-  } else if (tail == TAIL_ASG) {
-    if (st->done) return;
-    tail_assign(p);
-  } else if (tail == TAIL_COST) {
-    if (st->done) return;
-    tail_cost(p);
-  } else {
-    for (int e = threadIdx.x; e < p.k * p.d; e += blockDim.x) {
-      const int i = e / p.d, j = e - i * p.d;
-      p.med[e] = (double)p.mrows[(long long)st->mbest[i] * p.d + j];
-    }
-    __threadfence_block();
-    __syncthreads();
-    tail_refine(p);
-  }
+  if (tail != TAIL_REF && st->done) return;
+  TailMem T = tail_mem(p, smraw);
+  state_load(p, T.S);
+  if (tail == TAIL_LOC)
+    tail_locality(p, T);
+  else if (tail == TAIL_ASG)
+    tail_assign(p, T);
+  else if (tail == TAIL_COST)
+    tail_cost(p, T);
+  else
+    tail_refine(p, T);
+  state_store(p, T.S);
 }
 
-void launch_tail(const RunParams& p, int tail, cudaStream_t s) { k_tail<<<1, 256, 0, s>>>(p, tail); }
+void launch_tail(const RunParams& p, int tail, cudaStream_t s) {
+  k_tail<<<1, 256, p.tail_smem, s>>>(p, tail);
+}
 
 // ============================================================ shapes
 // Chunk P = 32 * PPT * NW points.  d <= 32: P = 256 (locality / labelsum 8
 // consumer warps x 1 point per lane, assign / final 4 warps x 2 points);
 // larger d: P = 128 or 64 so that the ring of (d + k) rows stays small.
-static size_t smem_loc(int P, int d, int k, int stages, int nw) {
-  CarveSize cs;
-  size_pipe(cs, d + k, P, stages, false);
-  cs.add<float>((size_t)k * d).add<ActSlot>(KMAX).add<int>(KMAX).add<double>(d);
-  cs.add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX);
-  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX).add<ExtraRows>(1);
-  return cs.s + 64;
-}
-static size_t smem_asg(int P, int d, int k, int stages, int nw) {
-  CarveSize cs;
-  size_pipe(cs, d, P, stages, false);
-  cs.add<float>((size_t)k * d).add<Term>((size_t)k * d).add<int>((size_t)k * d);
-  cs.add<int>(KMAX).add<int>(KMAX + 1).add<float>(KMAX).add<double>(d);
-  cs.add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX * 2);
-  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX);
-  return cs.s + 64;
-}
-static size_t smem_lsum(int P, int d, int k, int stages, int nw) {
-  CarveSize cs;
-  size_pipe(cs, d, P, stages, true);
-  cs.add<double>((size_t)k * d).add<int>((size_t)k * d).add<int>(KMAX).add<int>(KMAX + 1);
-  cs.add<double>(d).add<Cell>((size_t)k * d).add<unsigned>((size_t)nw * KMAX);
-  cs.add<long long>((size_t)nw * k * d).add<long long>((size_t)nw * KMAX);
-  return cs.s + 64;
-}
-static size_t smem_fin(int P, int d, int k, int stages) {
-  CarveSize cs;
-  size_pipe(cs, d, P, stages, false);
-  cs.add<float>((size_t)k * d).add<Term>((size_t)k * d).add<int>((size_t)k * d);
-  cs.add<int>(KMAX).add<float>(KMAX).add<double>(KMAX);
-  return cs.s + 64;
+struct LB {
+  size_t off = 0;
+  int take(size_t bytes) {
+    off = (off + 15) & ~(size_t)15;
+    const int r = (int)off;
+    off += bytes;
+    return r;
+  }
+};
+
+static SmemLayout blank_layout() {
+  SmemLayout L;
+  int* q = reinterpret_cast<int*>(&L);
+  for (size_t i = 0; i < sizeof(L) / sizeof(int); ++i) q[i] = -1;  // -1 = unused
+  return L;
 }
 
-PassShape pass_shape(int d, int k, int num_sms) {
+static TailLayout tail_layout(int d, int k, int nM) {
+  TailLayout t;
+  LB b;
+  const size_t kd = (size_t)k * d;
+  t.S = b.take(sizeof(DevState));
+  t.X = b.take(8 * kd);
+  t.Z = b.take(8 * kd);
+  t.med = b.take(8 * kd);
+  t.dev = b.take(8 * kd);
+  t.dm = b.take(kd);
+  t.pool = b.take(4 * (size_t)(nM > 0 ? nM : 1));
+  t.fnd = b.take(8 * 3 * KMAX);
+  t.bytes = (int)((b.off + 15) & ~(size_t)15);
+  return t;
+}
+
+static void finish(SmemLayout& L, LB& b, const TailLayout& tl) {
+  L.tail = L.buf;
+  size_t end = b.off;
+  if ((size_t)L.tail + tl.bytes > end) end = (size_t)L.tail + tl.bytes;
+  L.bytes = (int)((end + 64 + 15) & ~(size_t)15);
+}
+
+PassShape pass_shape(int d, int k, int nM, int num_sms) {
   PassShape ps;
   int P = 256, stages = 3;
   const int cfg[6][2] = {{256, 3}, {256, 2}, {128, 3}, {128, 2}, {64, 3}, {64, 2}};
@@ -1576,30 +1757,119 @@ PassShape pass_shape(int d, int k, int num_sms) {
   ps.tpb_asg = 32 * (nw2 + 1);
   ps.tpb_lsum = 32 * (nw1 + 1);
   ps.tpb_fin = 32 * (nw2 + 1);
-  ps.smem_loc = smem_loc(P, d, k, stages, nw1);
-  ps.smem_asg = smem_asg(P, d, k, stages, nw2);
-  ps.smem_cost = smem_lsum(P, d, k, stages, nw1);
+  const size_t kd = (size_t)k * d;
+  ps.tl = tail_layout(d, k, nM);
+  ps.tail_smem = ps.tl.bytes;
+  {  // locality
+    SmemLayout L = blank_layout();
+    LB b;
+    L.nw = nw1;
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * (d + k) * P * 4);
+    L.med = b.take(4 * (size_t)k * (d < 32 ? 32 : d));  // rows padded to 16 / 32
+    L.act = b.take(sizeof(ActSlot) * KMAX);
+    L.row = b.take(4 * KMAX);
+    L.scale = b.take(8 * (size_t)d);
+    L.cells = b.take(sizeof(Cell) * kd);
+    L.bal = b.take(4 * (size_t)nw1 * KMAX);
+    L.acc = b.take(8 * (size_t)nw1 * kd);
+    L.cnt = b.take(8 * (size_t)nw1 * KMAX);
+    L.ex = b.take(sizeof(ExtraRows));
+    L.thr = b.take(sizeof(Thr) * KMAX);
+    finish(L, b, ps.tl);
+    ps.lay[KK_LOC] = L;
+  }
+  {  // assign
+    SmemLayout L = blank_layout();
+    LB b;
+    L.nw = nw2;
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * d * P * 4);
+    L.med = b.take(4 * kd);
+    L.tab = b.take(sizeof(Term) * kd);
+    L.dl = b.take(4 * kd);
+    L.nD = b.take(4 * KMAX);
+    L.off = b.take(4 * (KMAX + 1));
+    L.rcp = b.take(4 * KMAX);
+    L.scale = b.take(8 * (size_t)d);
+    L.cells = b.take(sizeof(Cell) * kd);
+    L.bal = b.take(4 * (size_t)nw2 * KMAX * 2);
+    L.acc = b.take(8 * (size_t)nw2 * kd);
+    L.cnt = b.take(8 * (size_t)nw2 * KMAX);
+    finish(L, b, ps.tl);
+    ps.lay[KK_ASG] = L;
+  }
+  {  // labelsum (cost / refinement X)
+    SmemLayout L = blank_layout();
+    LB b;
+    L.nw = nw1;
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * d * P * 4);
+    L.lab = b.take((size_t)stages * P);
+    L.ctr = b.take(8 * kd);
+    L.dl = b.take(4 * kd);
+    L.nD = b.take(4 * KMAX);
+    L.off = b.take(4 * (KMAX + 1));
+    L.scale = b.take(8 * (size_t)d);
+    L.cells = b.take(sizeof(Cell) * kd);
+    L.bal = b.take(4 * (size_t)nw1 * KMAX);
+    L.acc = b.take(8 * (size_t)nw1 * kd);
+    L.cnt = b.take(8 * (size_t)nw1 * KMAX);
+    finish(L, b, ps.tl);
+    ps.lay[KK_LSUM] = L;
+  }
+  {  // final
+    SmemLayout L = blank_layout();
+    LB b;
+    L.nw = nw2;
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * d * P * 4);
+    L.med = b.take(4 * kd);
+    L.tab = b.take(sizeof(Term) * kd);
+    L.dl = b.take(4 * kd);
+    L.nD = b.take(4 * KMAX);
+    L.rcp = b.take(4 * KMAX);
+    L.Dl = b.take(8 * KMAX);
+    finish(L, b, ps.tl);
+    ps.lay[KK_FIN] = L;
+  }
+  ps.smem_loc = ps.lay[KK_LOC].bytes;
+  ps.smem_asg = ps.lay[KK_ASG].bytes;
+  ps.smem_cost = ps.lay[KK_LSUM].bytes;
   ps.smem_ref = ps.smem_cost;
-  ps.smem_fin = smem_fin(P, d, k, stages);
-  size_t mx = ps.smem_loc;
-  if (ps.smem_asg > mx) mx = ps.smem_asg;
-  if (ps.smem_cost > mx) mx = ps.smem_cost;
-  int per_sm = (int)((227 * 1024) / (mx + 1024));
-  if (per_sm < 1) per_sm = 1;
-  if (per_sm > 2048 / ps.tpb_loc) per_sm = 2048 / ps.tpb_loc;
-  if (per_sm > 8) per_sm = 8;
-  ps.per_sm = per_sm;
-  ps.grid = num_sms * per_sm;
+  ps.smem_fin = ps.lay[KK_FIN].bytes;
+  // persistent grids: as many resident blocks per SM as shared memory and
+  // the 2048-thread limit allow (<= 8), per kernel
+  auto grid_of = [&](size_t smem, int tpb) {
+    int per_sm = (int)((227 * 1024) / (smem + 1024));
+    if (per_sm > 2048 / tpb) per_sm = 2048 / tpb;
+    if (per_sm > 8) per_sm = 8;
+    if (per_sm < 1) per_sm = 1;
+    return num_sms * per_sm;
+  };
+  ps.grid_loc = grid_of(ps.smem_loc, ps.tpb_loc);
+  ps.grid_asg = grid_of(ps.smem_asg, ps.tpb_asg);
+  ps.grid_lsum = grid_of(ps.smem_cost, ps.tpb_lsum);
+  ps.grid_fin = grid_of(ps.smem_fin, ps.tpb_fin);
+  ps.grid = ps.grid_loc;
+  ps.per_sm = ps.grid_loc / num_sms;
   return ps;
 }
 
 cudaError_t configure_kernels(const PassShape& ps) {
   cudaError_t e;
-  const void* fns[] = {(const void*)k_locality<true>, (const void*)k_locality<false>,
-                       (const void*)k_assign<2>,       (const void*)k_labelsum<0>,
-                       (const void*)k_labelsum<1>,     (const void*)k_final<2>};
-  size_t sm[] = {ps.smem_loc, ps.smem_loc, ps.smem_asg, ps.smem_cost, ps.smem_ref, ps.smem_fin};
-  for (int i = 0; i < 6; ++i) {
+  const void* fns[] = {(const void*)k_locality<16>, (const void*)k_locality<32>,
+                       (const void*)k_locality<0>,  (const void*)k_assign<2>,
+                       (const void*)k_labelsum<0>,  (const void*)k_labelsum<1>,
+                       (const void*)k_final<2>,     (const void*)k_prepare,
+                       (const void*)k_tail};
+  const size_t sm[] = {ps.smem_loc,  ps.smem_loc, ps.smem_loc,   ps.smem_asg, ps.smem_cost,
+                       ps.smem_ref,  ps.smem_fin, (size_t)ps.tail_smem, (size_t)ps.tail_smem};
+  for (int i = 0; i < 9; ++i) {
     e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm[i]);
     if (e != cudaSuccess) return e;
   }
@@ -1607,22 +1877,24 @@ cudaError_t configure_kernels(const PassShape& ps) {
 }
 
 void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  if (p.d <= DREG)
-    k_locality<true><<<ps.grid, ps.tpb_loc, ps.smem_loc, s>>>(p);
+  if (p.d <= 16)
+    k_locality<16><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
+  else if (p.d <= 32)
+    k_locality<32><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
   else
-    k_locality<false><<<ps.grid, ps.tpb_loc, ps.smem_loc, s>>>(p);
+    k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_assign<2><<<ps.grid, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_labelsum<0><<<ps.grid, ps.tpb_lsum, ps.smem_cost, s>>>(p);
+  k_labelsum<0><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_cost, s>>>(p);
 }
 void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_labelsum<1><<<ps.grid, ps.tpb_lsum, ps.smem_ref, s>>>(p);
+  k_labelsum<1><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_ref, s>>>(p);
 }
 void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_final<2><<<ps.grid, ps.tpb_fin, ps.smem_fin, s>>>(p);
+  k_final<2><<<ps.grid_fin, ps.tpb_fin, ps.smem_fin, s>>>(p);
 }
 
 }  // namespace pc

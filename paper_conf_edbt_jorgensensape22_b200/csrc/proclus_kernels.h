@@ -13,9 +13,13 @@ struct PassShape {
   int P;          // points per chunk
   int stages;     // bulk-copy ring depth
   int tpb_loc, tpb_asg, tpb_lsum, tpb_fin;  // threads per block of each pass
-  int per_sm;     // resident blocks per SM
+  int per_sm;     // resident blocks per SM (locality)
   int grid;       // persistent blocks (SM count x per_sm)
+  int grid_loc, grid_asg, grid_lsum, grid_fin;  // per kernel
   size_t smem_loc, smem_asg, smem_cost, smem_ref, smem_fin;
+  SmemLayout lay[4];  // per KernelKind
+  TailLayout tl;
+  int tail_smem;
 };
 
 // N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value;
@@ -36,7 +40,7 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
 void launch_gather_m(const float* srows, const long long* sids, const int* spos, int nM, int d,
                      float* mrows, long long* mids, cudaStream_t s);
 
-PassShape pass_shape(int d, int k, int num_sms);
+PassShape pass_shape(int d, int k, int nM, int num_sms);
 cudaError_t configure_kernels(const PassShape& ps);
 
 // iteration prologue (delta, active slots) for the state's MCur
