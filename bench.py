@@ -195,8 +195,9 @@ def run_gpu(args):
     data, cfg = synth.config_data(args.config, seed=args.data_seed)
     n, d, k, l = cfg["n"], cfg["d"], cfg["k"], cfg["l"]
     metric = pk.METRIC_L2 if args.metric == "l2" else pk.METRIC_L1
-    lo = n * rank // world
-    hi = n * (rank + 1) // world
+    from paper_conf_edbt_jorgensensape22_b200.sharding import shard_rows
+
+    lo, hi = shard_rows(n, world, rank)  # boundaries on sub-chunk multiples
     shard = np.ascontiguousarray(data[lo:hi])
     uid = None
     if world > 1:
