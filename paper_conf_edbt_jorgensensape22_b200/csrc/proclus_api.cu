@@ -792,6 +792,11 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
       S.tail_ms[t] += (double)h->h_st->tail_ns[t] * 1e-6;
       S.fallbacks[t] += h->h_st->fallback[t];
     }
+    if (getenv("PROCLUS_TAIL_PROFILE")) {
+      fprintf(stderr, "tail_cycles");
+      for (int t = 0; t < 24; ++t) fprintf(stderr, " %llu", h->h_st->dbg_cyc[t]);
+      fprintf(stderr, "\n");
+    }
   }
   return PROCLUS_OK;
 }

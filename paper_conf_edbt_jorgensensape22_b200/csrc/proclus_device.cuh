@@ -46,6 +46,7 @@ struct DevState {
   double bytes_loc;             // algorithmic bytes of the locality passes
   long long fallback[4];        // exact fp64 re-decisions (loc, asg, fin, -)
   unsigned long long tail_ns[4];  // %globaltimer time in the single-block tails
+  unsigned long long dbg_cyc[24];  // per-phase SM cycles of the tails (PROCLUS_TAIL_PROFILE builds)
 };
 
 struct TraceBufs {
@@ -73,7 +74,9 @@ struct SmemLayout {
 };
 // Offsets (relative to SmemLayout::tail) of the single-block tail's scratch.
 struct TailLayout {
-  int S, X, Z, med, dev, dm, pool, fnd, bytes;
+  int S, X, Z, med, dev, dm, pool, fnd, isc, dl, dd;
+  int mrow, fall, uall, pall;  // rows of M and their tables, or mrow = -1
+  int bytes;
 };
 enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3 };
 

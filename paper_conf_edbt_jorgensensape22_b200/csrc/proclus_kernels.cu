@@ -25,6 +25,9 @@
 // graph while-node the cost tail also sets the loop condition.
 #include <math_constants.h>
 
+#include <cstdio>
+#include <cstdlib>
+
 #include "proclus_kernels.h"
 
 namespace pc {
@@ -159,7 +162,6 @@ void launch_gather_m(const float* srows, const long long* sids, const int* spos,
 // position, reading R7) with redux.sync on a 64-bit order key: 0 for picked
 // points, bits(dist) + 1 otherwise.
 constexpr int GR_TPB = 1024;
-constexpr int GR_PPT = 4;   // S-positions per thread in registers (nS <= 4096)
 
 __global__ void k_sdist(const float* __restrict__ srows, int nS, int d, int metric,
                         double* __restrict__ Ds) {
@@ -174,6 +176,359 @@ __global__ void k_sdist(const float* __restrict__ srows, int nS, int d, int metr
 struct KeyIdx {
   unsigned hi, lo, idx;
 };
+__device__ __forceinline__ KeyIdx warp_argmax(unsigned hi, unsigned lo, unsigned idx);
+__device__ __forceinline__ unsigned long long dkey(double v);
+
+// Cluster variant: the same picks spread over a thread-block cluster of CS
+// CTAs (one per SM), so the fp64 distance work of a pick runs on CS SMs.
+// Every CTA holds the whole sample in shared memory and owns positions
+// g, g + CS*GC_TPB, ... (g = rank*GC_TPB + tid).  Per pick each CTA reduces
+// each warp reduces its candidate and pushes it (16 bytes) into its slot of
+// every CTA of the cluster with st.async, completing 16 bytes of tx on the
+// receiver's mbarrier; a CTA proceeds when all CS*GC_W = 32 candidates landed
+// and reduces them with one warp argmax (slots parity double buffered: pick
+// i uses slot i&1).
+constexpr int GC_TPB = 64;
+constexpr int GC_W = GC_TPB / 32;
+
+__device__ __forceinline__ unsigned cluster_rank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::
+                   : "memory");
+}
+__device__ __forceinline__ unsigned mapa_u32(unsigned laddr, unsigned rank) {
+  unsigned r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(laddr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_async_v4(unsigned raddr, unsigned a, unsigned b, unsigned c,
+                                            unsigned d, unsigned rbar) {
+  asm volatile(
+      "st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, "
+      "[%5];" ::"r"(raddr),
+      "r"(a), "r"(b), "r"(c), "r"(d), "r"(rbar)
+      : "memory");
+}
+
+// Distances of the owned positions to pick qs: DP > 0 is d rounded up to a
+// multiple of 8 (zero-padded dimensions add exact zeros to the oracle-order
+// sum, so the result is unchanged) and fully unrolled; DP = 0 loops over d.
+template <int NP, int METRIC, int CS, int DP>
+__device__ __forceinline__ void greedy_update_c(const double* __restrict__ gT, int nSp, int nS,
+                                                int d, int g, int qs, bool first,
+                                                double (&dreg)[NP]) {
+  constexpr int STRIDE = CS * GC_TPB;
+  double acc[NP];
+#pragma unroll
+  for (int t = 0; t < NP; ++t) acc[t] = 0.0;
+  if (DP > 0) {
+#pragma unroll
+    for (int j = 0; j < DP; ++j) {
+      const double pj = gT[j * nSp + qs];
+#pragma unroll
+      for (int t = 0; t < NP; ++t) {
+        const double df = dsub(gT[j * nSp + g + t * STRIDE], pj);
+        acc[t] = dadd(acc[t], METRIC == 1 ? fabs(df) : dmul(df, df));
+      }
+    }
+  } else {
+    for (int j = 0; j < d; ++j) {
+      const double pj = gT[j * nSp + qs];
+#pragma unroll
+      for (int t = 0; t < NP; ++t) {
+        const double df = dsub(gT[j * nSp + g + t * STRIDE], pj);
+        acc[t] = dadd(acc[t], METRIC == 1 ? fabs(df) : dmul(df, df));
+      }
+    }
+  }
+#pragma unroll
+  for (int t = 0; t < NP; ++t) {
+    const int q = g + t * STRIDE;
+    const double u = METRIC == 1 ? acc[t] : __dsqrt_rn(acc[t]);
+    if (first) {
+      dreg[t] = (q < nS && q != qs) ? u : -1.0;
+    } else if (q == qs) {
+      dreg[t] = -1.0;
+    } else if (dreg[t] >= 0.0 && u < dreg[t]) {
+      dreg[t] = u;
+    }
+  }
+}
+
+// Sample rows [nS][d] fp32 -> [dp][nSp] fp64 (zero padded), the layout the
+// cluster greedy copies into each CTA's shared memory with bulk copies.
+__global__ void k_sample_soa(const float* __restrict__ srows, int nS, int d, int dp, int nSp,
+                             double* __restrict__ out) {
+  const int tot = dp * nSp;
+  for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < tot; e += gridDim.x * blockDim.x) {
+    const int j = e / nSp, q = e - j * nSp;
+    out[e] = (q < nS && j < d) ? (double)srows[(long long)q * d + j] : 0.0;
+  }
+}
+
+template <int NP, int METRIC, int CS, int DP>
+__global__ void __launch_bounds__(GC_TPB)
+    k_greedy_cluster(const double* __restrict__ sT, int nS, int d, int dp, int nM, int q0,
+                     int* __restrict__ spos, double* __restrict__ pickdist) {
+  extern __shared__ __align__(16) double gT[];  // [dp][nSp], nSp = NP * CS * GC_TPB
+  static_assert(CS * GC_W == 32, "one candidate slot per lane");
+  __shared__ __align__(16) unsigned cand[2][CS * GC_W][4];
+  __shared__ __align__(8) unsigned long long bar[3];
+  constexpr int nSp = NP * CS * GC_TPB;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const unsigned rank = cluster_rank();
+  const int g = (int)rank * GC_TPB + tid;
+  if (tid == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    mbar_init(&bar[2], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (tid == 0) {  // the whole sample: bulk copies of <= 32 KB on bar[2]
+    const unsigned bytes = (unsigned)(sizeof(double) * (size_t)dp * nSp);
+    mbar_expect_tx(&bar[2], bytes);
+    for (unsigned off = 0; off < bytes; off += 32768u) {
+      const unsigned len = bytes - off < 32768u ? bytes - off : 32768u;
+      bulk_g2s((char*)gT + off, (const char*)sT + off, len, &bar[2]);
+    }
+  }
+  cluster_sync_all();  // every CTA's barriers are initialised before any push
+  mbar_wait(&bar[2], 0u);
+  double dreg[NP];
+  greedy_update_c<NP, METRIC, CS, DP>(gT, nSp, nS, d, g, q0, true, dreg);
+  if (rank == 0 && tid == 0) {
+    spos[0] = q0;
+    if (pickdist) pickdist[0] = CUDART_INF;
+  }
+  for (int i = 1; i < nM; ++i) {
+    const int par = i & 1;
+    const unsigned ph = (unsigned)(((i - 1) >> 1) & 1);  // use count of slot par
+    if (tid == 0) mbar_expect_tx(&bar[par], CS * GC_W * 16u);
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const unsigned long long key = dkey(dreg[t]);
+      if (key > bk) {
+        bk = key;
+        bq = g + t * CS * GC_TPB;
+      }
+    }
+    // every warp pushes its candidate into slot (rank, w) of every CTA
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    if (lane < CS)
+      st_async_v4(mapa_u32(smem_u32(&cand[par][rank * GC_W + w][0]), (unsigned)lane), r.hi, r.lo,
+                  r.idx, 0u, mapa_u32(smem_u32(&bar[par]), (unsigned)lane));
+    mbar_wait(&bar[par], ph);
+    KeyIdx s = warp_argmax(cand[par][lane][0], cand[par][lane][1], cand[par][lane][2]);
+    const int qs = (int)s.idx;
+    if (rank == 0 && tid == 0) {
+      spos[i] = qs;
+      if (pickdist) {
+        unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
+        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+      }
+    }
+    if (i + 1 < nM) greedy_update_c<NP, METRIC, CS, DP>(gT, nSp, nS, d, g, qs, false, dreg);
+  }
+  cluster_sync_all();  // no CTA leaves while a peer may still push into it
+}
+
+
+// Greedy with the sample resident in shared memory, transposed to [j][q]
+// (fp64, zero padded to NP*256 positions): every pick recomputes the
+// distances of the NP owned positions to the new medoid in registers.  The d
+// per-dimension terms are formed four at a time ahead of the oracle-order
+// chain of additions (j ascending), so only the dadd chain is serial.  One
+// barrier per pick and a redundant 8-way argmax.
+template <int NP, int METRIC>
+__device__ __forceinline__ void greedy_update(const double* __restrict__ gT, int nSp, int nS,
+                                              int d, int qs, bool first, double (&dreg)[NP]) {
+  const int tid = threadIdx.x;
+  double acc[NP];
+#pragma unroll
+  for (int t = 0; t < NP; ++t) acc[t] = 0.0;
+  int j = 0;
+  for (; j + 4 <= d; j += 4) {
+    double pj[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) pj[u] = gT[(j + u) * nSp + qs];
+    double tm[NP][4];
+#pragma unroll
+    for (int t = 0; t < NP; ++t)
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const double df = dsub(gT[(j + u) * nSp + tid + t * 256], pj[u]);
+        tm[t][u] = METRIC == 1 ? fabs(df) : dmul(df, df);
+      }
+#pragma unroll
+    for (int t = 0; t < NP; ++t)
+      acc[t] = dadd(dadd(dadd(dadd(acc[t], tm[t][0]), tm[t][1]), tm[t][2]), tm[t][3]);
+  }
+  for (; j < d; ++j) {
+    const double pj = gT[j * nSp + qs];
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const double df = dsub(gT[j * nSp + tid + t * 256], pj);
+      acc[t] = dadd(acc[t], METRIC == 1 ? fabs(df) : dmul(df, df));
+    }
+  }
+#pragma unroll
+  for (int t = 0; t < NP; ++t) {
+    const int q = tid + t * 256;
+    const double u = METRIC == 1 ? acc[t] : __dsqrt_rn(acc[t]);
+    if (first) {
+      dreg[t] = (q < nS && q != qs) ? u : -1.0;
+    } else if (q == qs) {
+      dreg[t] = -1.0;
+    } else if (dreg[t] >= 0.0 && u < dreg[t]) {
+      dreg[t] = u;
+    }
+  }
+}
+
+template <int NP, int METRIC>
+__global__ void __launch_bounds__(256)
+    k_greedy_smem(const float* __restrict__ srows, int nS, int d, int nM, int q0,
+                  int* __restrict__ spos, double* __restrict__ pickdist) {
+  extern __shared__ double gT[];  // [d][NP*256]
+  __shared__ unsigned whi[2][8], wlo[2][8], widx[2][8];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  constexpr int nSp = NP * 256;
+  for (int e = tid; e < nSp * d; e += 256) {
+    const int j = e / nSp, q = e - j * nSp;
+    gT[e] = q < nS ? (double)srows[(long long)q * d + j] : 0.0;
+  }
+  __syncthreads();
+  double dreg[NP];
+  greedy_update<NP, METRIC>(gT, nSp, nS, d, q0, true, dreg);
+  if (tid == 0) {
+    spos[0] = q0;
+    if (pickdist) pickdist[0] = CUDART_INF;
+  }
+  for (int i = 1; i < nM; ++i) {
+    // pick i: argmax over unpicked (larger distance, then smaller position)
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const unsigned long long key = dkey(dreg[t]);
+      if (key > bk) {
+        bk = key;
+        bq = tid + t * 256;
+      }
+    }
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    const int par = i & 1;
+    if (lane == 0) {
+      whi[par][w] = r.hi;
+      wlo[par][w] = r.lo;
+      widx[par][w] = r.idx;
+    }
+    __syncthreads();
+    KeyIdx s = warp_argmax(lane < 8 ? whi[par][lane] : 0u, lane < 8 ? wlo[par][lane] : 0u,
+                           lane < 8 ? widx[par][lane] : 0xffffffffu);
+    const int qs = (int)s.idx;
+    if (tid == 0) {
+      spos[i] = qs;
+      if (pickdist) {
+        unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
+        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+      }
+    }
+    if (i + 1 < nM) greedy_update<NP, METRIC>(gT, nSp, nS, d, qs, false, dreg);
+  }
+}
+
+__device__ __forceinline__ KeyIdx warp_argmax(unsigned hi, unsigned lo, unsigned idx);
+__device__ __forceinline__ unsigned long long dkey(double v);
+
+// Greedy with the sample rows resident in shared memory (fp64): every pick
+// recomputes the distances of the owned positions to the new medoid in
+// registers (NP positions per thread, the j loop outside so the NP oracle-
+// order chains interleave), then one barrier and a redundant 8-way argmax.
+template <int NP>
+__global__ void __launch_bounds__(256)
+    k_greedy_smem(const float* __restrict__ srows, int nS, int d, int nM, int q0, int metric,
+                  int* __restrict__ spos, double* __restrict__ pickdist) {
+  extern __shared__ double grows[];  // [nS][d]
+  __shared__ unsigned whi[2][8], wlo[2][8], widx[2][8];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  for (int e = tid; e < nS * d; e += 256) grows[e] = (double)srows[e];
+  __syncthreads();
+  double dreg[NP];
+  // distances of the owned positions to pick qs (oracle order, j ascending)
+  auto update = [&](int qs, bool first) {
+    double acc[NP];
+#pragma unroll
+    for (int t = 0; t < NP; ++t) acc[t] = 0.0;
+    const double* pr = grows + (long long)qs * d;
+    for (int j = 0; j < d; ++j) {
+      const double pj = pr[j];
+#pragma unroll
+      for (int t = 0; t < NP; ++t) {
+        const int q = tid + t * 256;
+        const double x = q < nS ? grows[(long long)q * d + j] : 0.0;
+        const double df = dsub(x, pj);
+        acc[t] = metric == 1 ? dadd(acc[t], fabs(df)) : dadd(acc[t], dmul(df, df));
+      }
+    }
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const int q = tid + t * 256;
+      const double u = metric == 1 ? acc[t] : __dsqrt_rn(acc[t]);
+      if (first) {
+        dreg[t] = (q < nS && q != qs) ? u : -1.0;
+      } else if (q == qs) {
+        dreg[t] = -1.0;
+      } else if (dreg[t] >= 0.0 && u < dreg[t]) {
+        dreg[t] = u;
+      }
+    }
+  };
+  update(q0, true);
+  if (tid == 0) {
+    spos[0] = q0;
+    if (pickdist) pickdist[0] = CUDART_INF;
+  }
+  for (int i = 1; i < nM; ++i) {
+    // pick i: argmax over unpicked (larger distance, then smaller position)
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const unsigned long long key = dkey(dreg[t]);
+      if (key > bk) {
+        bk = key;
+        bq = tid + t * 256;
+      }
+    }
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    const int par = i & 1;
+    if (lane == 0) {
+      whi[par][w] = r.hi;
+      wlo[par][w] = r.lo;
+      widx[par][w] = r.idx;
+    }
+    __syncthreads();
+    KeyIdx s = warp_argmax(lane < 8 ? whi[par][lane] : 0u, lane < 8 ? wlo[par][lane] : 0u,
+                           lane < 8 ? widx[par][lane] : 0xffffffffu);
+    const int qs = (int)s.idx;
+    if (tid == 0) {
+      spos[i] = qs;
+      if (pickdist) {
+        unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
+        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+      }
+    }
+    if (i + 1 < nM) update(qs, false);
+  }
+}
 
 __device__ __forceinline__ KeyIdx warp_argmax(unsigned hi, unsigned lo, unsigned idx) {
   const unsigned full = 0xffffffffu;
@@ -314,11 +669,102 @@ __global__ void __launch_bounds__(GR_TPB)
 }
 
 size_t greedy_scratch_doubles(int nS) {
-  return nS <= GM_PPT * GM_TPB ? (size_t)nS * nS : (size_t)nS;
+  // distance matrix (k_greedy), or the fp64 SoA sample of the cluster greedy
+  const size_t m = nS <= GM_PPT * GM_TPB ? (size_t)nS * nS : (size_t)nS;
+  const size_t soa = (size_t)32 * 4 * 16 * 64;
+  return m > soa ? m : soa;
+}
+
+template <int NP>
+static cudaError_t greedy_smem_launch(const float* srows, int nS, int d, int nM, int q0,
+                                      int metric, int* spos, double* pickdist, cudaStream_t s) {
+  const size_t bytes = sizeof(double) * (size_t)NP * 256 * d;
+  cudaError_t e;
+  if (metric == 1) {
+    e = cudaFuncSetAttribute(k_greedy_smem<NP, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)bytes);
+    if (e == cudaSuccess)
+      k_greedy_smem<NP, 1><<<1, 256, bytes, s>>>(srows, nS, d, nM, q0, spos, pickdist);
+  } else {
+    e = cudaFuncSetAttribute(k_greedy_smem<NP, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)bytes);
+    if (e == cudaSuccess)
+      k_greedy_smem<NP, 0><<<1, 256, bytes, s>>>(srows, nS, d, nM, q0, spos, pickdist);
+  }
+  if (e != cudaSuccess) return e;
+  return cudaGetLastError();
+}
+
+template <int NP, int METRIC, int DP>
+static cudaError_t greedy_cluster_launch(const double* sT, int nS, int d, int dp, int nM, int q0,
+                                         int* spos, double* pickdist, cudaStream_t s) {
+  constexpr int CS = 16;
+  const size_t bytes = sizeof(double) * (size_t)NP * CS * GC_TPB * dp;
+  auto fn = k_greedy_cluster<NP, METRIC, CS, DP>;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(CS, 1, 1);
+  cfg.blockDim = dim3(GC_TPB, 1, 1);
+  cfg.dynamicSmemBytes = bytes;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = CS;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, fn, sT, nS, d, dp, nM, q0, spos, pickdist);
+}
+
+template <int NP, int DP>
+static cudaError_t greedy_cluster_m(const double* sT, int nS, int d, int dp, int nM, int q0,
+                                    int metric, int* spos, double* pickdist, cudaStream_t s) {
+  return metric == 1
+             ? greedy_cluster_launch<NP, 1, DP>(sT, nS, d, dp, nM, q0, spos, pickdist, s)
+             : greedy_cluster_launch<NP, 0, DP>(sT, nS, d, dp, nM, q0, spos, pickdist, s);
+}
+
+template <int NP>
+static cudaError_t greedy_cluster_np(const double* sT, int nS, int d, int dp, int nM, int q0,
+                                     int metric, int* spos, double* pickdist, cudaStream_t s) {
+  switch (dp) {
+    case 8: return greedy_cluster_m<NP, 8>(sT, nS, d, dp, nM, q0, metric, spos, pickdist, s);
+    case 16: return greedy_cluster_m<NP, 16>(sT, nS, d, dp, nM, q0, metric, spos, pickdist, s);
+    case 32: return greedy_cluster_m<NP, 32>(sT, nS, d, dp, nM, q0, metric, spos, pickdist, s);
+    default: return greedy_cluster_m<NP, 0>(sT, nS, d, dp, nM, q0, metric, spos, pickdist, s);
+  }
 }
 
 cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
                           double* scratch, int* spos, double* pickdist, cudaStream_t s) {
+  {  // cluster of 16 CTAs x 64 threads: NP positions per thread
+    const int per = 16 * GC_TPB;
+    const int npc = nS <= per ? 1 : nS <= 2 * per ? 2 : nS <= 4 * per ? 4 : 0;
+    const int dp = d <= 8 ? 8 : d <= 16 ? 16 : d <= 32 ? 32 : ((d + 1) / 2) * 2;
+    const size_t soa = (size_t)dp * npc * per;  // doubles
+    if (npc && sizeof(double) * soa <= 200 * 1024 && soa <= greedy_scratch_doubles(nS) &&
+        !getenv("PROCLUS_GREEDY_1CTA")) {
+      k_sample_soa<<<(int)((soa + 255) / 256), 256, 0, s>>>(srows, nS, d, dp, npc * per, scratch);
+      cudaError_t e = npc == 1 ? greedy_cluster_np<1>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
+                      : npc == 2 ? greedy_cluster_np<2>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
+                                 : greedy_cluster_np<4>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s);
+      if (e == cudaSuccess) return cudaSuccess;
+      cudaGetLastError();  // cluster launch unavailable: single-CTA kernels below
+    }
+  }
+  const int np = nS <= 256 ? 1 : nS <= 512 ? 2 : nS <= 1024 ? 4 : nS <= 2048 ? 8 : 16;
+  if (nS <= 16 * 256 && sizeof(double) * (size_t)np * 256 * d <= 200 * 1024) {
+    switch (np) {
+      case 1: return greedy_smem_launch<1>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
+      case 2: return greedy_smem_launch<2>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
+      case 4: return greedy_smem_launch<4>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
+      case 8: return greedy_smem_launch<8>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
+      default: return greedy_smem_launch<16>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
+    }
+  }
   if (nS <= GM_PPT * GM_TPB) {
     const long long tot = (long long)nS * nS;
     int blocks = (int)((tot + 255) / 256);
@@ -379,10 +825,10 @@ __device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
   const unsigned row = (unsigned)p.P * 4u;
   const int nex = ex ? ex->n : 0;
   const unsigned bytes = row * (unsigned)(p.d + nex) + (labsrc ? (unsigned)p.P : 0u);
+  int stg = 0, round = 0;
   for (long long i = 0; i < nmy; ++i) {
-    const int stg = (int)(i % p.stages);
-    if (i >= p.stages) {  // the consumers of chunk i - stages released this stage
-      mbar_wait(&R.empty[stg], (unsigned)(((i / p.stages) - 1) & 1));
+    if (round > 0) {  // the consumers of chunk i - stages released this stage
+      mbar_wait(&R.empty[stg], (unsigned)((round - 1) & 1));
       fence_proxy_async();
     }
     const long long base = (blockIdx.x + i * gridDim.x) * (long long)p.P;
@@ -395,8 +841,25 @@ __device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
     }
     if (labsrc && lane == 0)
       bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, &R.full[stg]);
+    if (++stg == p.stages) {
+      stg = 0;
+      ++round;
+    }
   }
 }
+
+// Consumer-side ring position: stage index and the parity of its full
+// barrier, advanced without integer division.
+struct RingPos {
+  int stg = 0;
+  unsigned ph = 0;
+  __device__ __forceinline__ void next(int stages) {
+    if (++stg == stages) {
+      stg = 0;
+      ph ^= 1u;
+    }
+  }
+};
 
 __device__ __forceinline__ void pipe_release(const Pipe& R, int stg) {
   __syncwarp();
@@ -552,10 +1015,6 @@ __device__ Pipe carve_pipe(Carve& cv, const RunParams& p, int rows, bool with_la
   R.lab = with_lab ? cv.take<unsigned char>((size_t)p.stages * p.P) : nullptr;
   return R;
 }
-static void size_pipe(CarveSize& cs, int rows, int P, int stages, bool with_lab) {
-  cs.add<unsigned long long>(SMAX).add<unsigned long long>(SMAX).add<float>((size_t)stages * rows * P);
-  if (with_lab) cs.add<unsigned char>((size_t)stages * P);
-}
 
 // ============================================================ certified tests
 // The fp32 value f approximates the oracle's fp64 value v with
@@ -633,18 +1092,52 @@ __device__ __noinline__ int exact_argmin(const float* __restrict__ x, int P,
 
 // ============================================================ tails
 // The single-block steps between passes run on a shared-memory copy of the
-// device state (DevState) and of every small array they touch; global memory
-// is read in parallel at the start and written in parallel at the end, so no
-// thread waits on a chain of dependent global loads.
+// device state (DevState) and of every small array they touch.  They are
+// latency-bound (a few hundred values), so each tail is organised in as few
+// global-memory round trips as possible: the independent loads (state words,
+// accumulators, small tables) are all issued before the first one is used,
+// and the serial logic runs on warps with ballots / redux instead of single
+// threads walking shared memory.
+#ifdef PROCLUS_TAIL_PROFILE
+__shared__ unsigned long long g_tst_last;
+#define TST_START()                                        \
+  do {                                                     \
+    if (threadIdx.x == 0) g_tst_last = clock64();          \
+  } while (0)
+#define TST(T, idx)                                        \
+  do {                                                     \
+    __syncthreads();                                       \
+    if (threadIdx.x == 0) {                                \
+      const unsigned long long t_ = clock64();             \
+      (T).S->dbg_cyc[idx] += t_ - g_tst_last;              \
+      g_tst_last = t_;                                     \
+    }                                                      \
+  } while (0)
+#else
+#define TST_START() \
+  do {              \
+  } while (0)
+#define TST(T, idx) \
+  do {              \
+  } while (0)
+#endif
+
 struct TailMem {
   DevState* S;
-  double* X;      // [k*d]
-  double* Z;      // [k*d]
-  double* med;    // [k*d] medoid rows, fp64
-  double* dev;    // [k*d]
+  double* X;          // [k*d]
+  double* Z;          // [k*d] (also raw accumulator values before Z exists)
+  double* med;        // [k*d] medoid rows, fp64
+  double* dev;        // [k*d] (also H rows / selection keys)
   unsigned char* dm;  // [k*d]
-  int* pool;      // [nM]
-  double* fnd;    // [3*KMAX]: found / used / delta' of the current slots
+  int* pool;          // [nM]
+  double* fnd;        // [3*KMAX]: found / used / delta' of the current slots
+  double* isc;        // [d] 2^-e_j
+  int* dl;            // [k*d] dimension lists
+  double* dd;         // [k*k] medoid distances
+  float* mrow;        // [nM*d] rows of M, or nullptr (not cached)
+  unsigned char* fall;  // [nM] DistFound of M (with mrow)
+  unsigned char* uall;  // [nM] delta' valid
+  double* pall;         // [nM] delta'
 };
 
 __device__ __forceinline__ TailMem tail_mem(const RunParams& p, unsigned char* base) {
@@ -658,46 +1151,108 @@ __device__ __forceinline__ TailMem tail_mem(const RunParams& p, unsigned char* b
   T.dm = base + t.dm;
   T.pool = (int*)(base + t.pool);
   T.fnd = (double*)(base + t.fnd);
+  T.isc = (double*)(base + t.isc);
+  T.dl = (int*)(base + t.dl);
+  T.dd = (double*)(base + t.dd);
+  T.mrow = t.mrow >= 0 ? (float*)(base + t.mrow) : nullptr;
+  T.fall = t.mrow >= 0 ? base + t.fall : nullptr;
+  T.uall = t.mrow >= 0 ? base + t.uall : nullptr;
+  T.pall = t.mrow >= 0 ? (double*)(base + t.pall) : nullptr;
   return T;
 }
 
-__device__ void state_load(const RunParams& p, DevState* S) {
+// DevState words in registers: issue() starts the loads, commit() stores them
+// into the shared copy, so their latency overlaps the loads in between.
+constexpr int STATE_WORDS = (int)(sizeof(DevState) / 4);
+constexpr int STATE_REGS = 8;  // words in flight per thread; the rest is copied in commit()
+struct StateRegs {
+  unsigned v[STATE_REGS];
+};
+__device__ __forceinline__ void state_issue(const RunParams& p, StateRegs& r) {
   const unsigned* src = (const unsigned*)p.st;
+#pragma unroll
+  for (int q = 0; q < STATE_REGS; ++q) {
+    const int i = threadIdx.x + q * blockDim.x;
+    r.v[q] = i < STATE_WORDS ? __ldcg(src + i) : 0u;
+  }
+}
+__device__ __forceinline__ void state_commit(const RunParams& p, const StateRegs& r, DevState* S) {
   unsigned* dst = (unsigned*)S;
-  for (int i = threadIdx.x; i < (int)(sizeof(DevState) / 4); i += blockDim.x) dst[i] = __ldcg(src + i);
+#pragma unroll
+  for (int q = 0; q < STATE_REGS; ++q) {
+    const int i = threadIdx.x + q * blockDim.x;
+    if (i < STATE_WORDS) dst[i] = r.v[q];
+  }
+  const unsigned* src = (const unsigned*)p.st;  // small blocks: the remainder
+  for (int i = threadIdx.x + STATE_REGS * blockDim.x; i < STATE_WORDS; i += blockDim.x)
+    dst[i] = __ldcg(src + i);
+}
+__device__ void state_load(const RunParams& p, DevState* S) {
+  StateRegs r;
+  state_issue(p, r);
+  state_commit(p, r, S);
   __syncthreads();
 }
 __device__ void state_store(const RunParams& p, const DevState* S) {
   __syncthreads();
   const unsigned* src = (const unsigned*)S;
   unsigned* dst = (unsigned*)p.st;
-  for (int i = threadIdx.x; i < (int)(sizeof(DevState) / 4); i += blockDim.x) dst[i] = src[i];
+  for (int i = threadIdx.x; i < STATE_WORDS; i += blockDim.x) dst[i] = src[i];
+}
+
+// Warp argmin of (key, j) over keys[0..d) skipping j == excl: smallest key,
+// then smaller j.  Every lane returns the winning j.
+__device__ __forceinline__ int warp_argmin_row(const unsigned long long* keys, int d, int excl) {
+  const int lane = threadIdx.x & 31;
+  unsigned long long bk = ~0ull;
+  unsigned bj = 0xffffffffu;
+  for (int j = lane; j < d; j += 32) {
+    const unsigned long long kj = keys[j];
+    if (j != excl && kj < bk) {  // ascending j per lane: strict < keeps the smaller j
+      bk = kj;
+      bj = (unsigned)j;
+    }
+  }
+  const unsigned full = 0xffffffffu;
+  const unsigned hi = (unsigned)(bk >> 32), lo = (unsigned)bk;
+  const unsigned mhi = __reduce_min_sync(full, hi);
+  const unsigned mlo = __reduce_min_sync(full, hi == mhi ? lo : 0xffffffffu);
+  return (int)__reduce_min_sync(full, (hi == mhi && lo == mlo) ? bj : 0xffffffffu);
 }
 
 // ------------------------------------------------------------ FindDimensions
 // Y_i, sigma_i, Z_ij (Alg 4 l.6-13, readings R2, R3) and the
 // selection of Alg 4 l.15-16 (reading R10): per medoid the two smallest by
-// (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j), found with a
-// block-wide radix select on order-preserving keys.  All in shared memory;
-// writes D as a mask (T.dm), |D_i| (S->nD) and, in global memory, the mask
-// and the ascending dimension lists used by the passes.
+// (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j).  The order is
+// taken on order-preserving 64-bit keys of Z (T.dev); the rest is selected by
+// rank (each free cell counts the free cells before it) when k*d <= 2048,
+// else by a block-wide radix select.  Writes D as a mask (T.dm), |D_i|
+// (S->nD) and, in global memory, the mask and the ascending dimension lists
+// used by the passes.  Needs X in T.X; clobbers T.Z and T.dev.
 __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   __shared__ double Ys[KMAX], Ss[KMAX];
-  __shared__ unsigned int hist[256];
-  __shared__ unsigned long long prefix_s;
-  __shared__ int need_s;
-  __shared__ int tcount[TPB_MAX];
-  const int tid = threadIdx.x, bd = blockDim.x;
+  const int tid = threadIdx.x, bd = blockDim.x, lane = tid & 31, w = tid >> 5, nw = bd >> 5;
   const int k = p.k, d = p.d, l = p.l, kd = k * d;
   const double* X = T.X;
   double* Z = T.Z;
   unsigned char* dm = T.dm;
-  if (tid < k) {
+  unsigned long long* key = (unsigned long long*)T.dev;
+  if (tid < k) {  // oracle order: j ascending, four loads in flight
     const double* x = X + tid * d;
     double Y = 0.0, s2 = 0.0;
-    for (int j = 0; j < d; ++j) Y = dadd(Y, x[j]);
+    int j = 0;
+    for (; j + 4 <= d; j += 4) {
+      const double a = x[j], b = x[j + 1], c = x[j + 2], e = x[j + 3];
+      Y = dadd(dadd(dadd(dadd(Y, a), b), c), e);
+    }
+    for (; j < d; ++j) Y = dadd(Y, x[j]);
     Y = ddiv(Y, (double)d);
-    for (int j = 0; j < d; ++j) {
+    for (j = 0; j + 4 <= d; j += 4) {
+      const double a = dsub(x[j], Y), b = dsub(x[j + 1], Y), c = dsub(x[j + 2], Y),
+                   e = dsub(x[j + 3], Y);
+      s2 = dadd(dadd(dadd(dadd(s2, dmul(a, a)), dmul(b, b)), dmul(c, c)), dmul(e, e));
+    }
+    for (; j < d; ++j) {
       const double u = dsub(x[j], Y);
       s2 = dadd(s2, dmul(u, u));
     }
@@ -705,27 +1260,53 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     Ss[tid] = __dsqrt_rn(ddiv(s2, (double)(d - 1)));
   }
   __syncthreads();
+  TST(T, 2);
   for (int c = tid; c < kd; c += bd) {
     const int i = c / d;
     const double sg = Ss[i];
-    Z[c] = (sg == 0.0) ? 0.0 : ddiv(dsub(X[c], Ys[i]), sg);
+    const double z = (sg == 0.0) ? 0.0 : ddiv(dsub(X[c], Ys[i]), sg);
+    Z[c] = z;
+    key[c] = sortable_key(z);
     dm[c] = 0;
   }
   __syncthreads();
-  if (tid < k) {  // two smallest per row, ties -> smaller j
-    const double* z = Z + tid * d;
-    int j1 = 0;
-    for (int j = 1; j < d; ++j)
-      if (z[j] < z[j1]) j1 = j;
-    int j2 = (j1 == 0) ? 1 : 0;
-    for (int j = 0; j < d; ++j)
-      if (j != j1 && z[j] < z[j2]) j2 = j;
-    dm[tid * d + j1] = 1;
-    dm[tid * d + j2] = 1;
+  TST(T, 3);
+  for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
+    const int j1 = warp_argmin_row(key + i * d, d, -1);
+    const int j2 = warp_argmin_row(key + i * d, d, j1);
+    if (lane == 0) {
+      dm[i * d + j1] = 1;
+      dm[i * d + j2] = 1;
+    }
   }
   __syncthreads();
+  TST(T, 4);
   const int R = k * l - 2 * k;
-  if (R > 0) {
+  if (R > 0 && kd <= 2048) {
+    for (int c = tid; c < kd; c += bd)
+      if (dm[c]) key[c] = ~0ull;  // taken: never before a free cell
+    __syncthreads();
+    for (int c = tid; c < kd; c += bd) {
+      if (dm[c]) continue;
+      const unsigned long long kc = key[c];
+      int rank = 0;
+      int o = 0;
+      for (; o + 4 <= kd; o += 4) {
+        const unsigned long long k0 = key[o], k1 = key[o + 1], k2 = key[o + 2], k3 = key[o + 3];
+        rank += (k0 < kc || (k0 == kc && o < c)) + (k1 < kc || (k1 == kc && o + 1 < c)) +
+                (k2 < kc || (k2 == kc && o + 2 < c)) + (k3 < kc || (k3 == kc && o + 3 < c));
+      }
+      for (; o < kd; ++o) {
+        const unsigned long long ko = key[o];
+        rank += (ko < kc || (ko == kc && o < c));
+      }
+      if (rank < R) dm[c] = 1;
+    }
+  } else if (R > 0) {
+    __shared__ unsigned int hist[256];
+    __shared__ unsigned long long prefix_s;
+    __shared__ int need_s;
+    __shared__ int tcount[TPB_MAX];
     if (tid == 0) {
       prefix_s = 0ull;
       need_s = R;
@@ -737,8 +1318,8 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
       const unsigned long long pre = prefix_s;
       for (int c = tid; c < kd; c += bd) {
         if (dm[c]) continue;
-        const unsigned long long key = sortable_key(Z[c]);
-        if ((key & hmask) == pre) atomicAdd(&hist[(key >> shift) & 255ull], 1u);
+        const unsigned long long kc = key[c];
+        if ((kc & hmask) == pre) atomicAdd(&hist[(kc >> shift) & 255ull], 1u);
       }
       __syncthreads();
       if (tid < 32) {  // warp scan over 256 bins, 8 per lane
@@ -778,7 +1359,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     const int c0 = tid * per, c1 = min(kd, c0 + per);
     int eq = 0;
     for (int c = c0; c < c1; ++c)
-      if (!dm[c] && sortable_key(Z[c]) == K) ++eq;
+      if (!dm[c] && key[c] == K) ++eq;
     tcount[tid] = eq;
     __syncthreads();
     if (tid < 32) {  // exclusive scan of tcount[0..bd) by one warp
@@ -799,60 +1380,78 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     int rank = tcount[tid];
     for (int c = c0; c < c1; ++c) {  // own contiguous range only
       if (dm[c]) continue;
-      const unsigned long long key = sortable_key(Z[c]);
-      if (key < K || (key == K && rank++ < need)) dm[c] = 1;
+      const unsigned long long kc = key[c];
+      if (kc < K || (kc == K && rank++ < need)) dm[c] = 1;
     }
   }
   __syncthreads();
-  if (tid < k) {  // |D_i| and the ascending lists (global, for the passes)
-    int t = 0;
-    for (int j = 0; j < d; ++j)
-      if (dm[tid * d + j]) p.dlist[tid * d + t++] = j;
-    T.S->nD[tid] = t;
+  TST(T, 6);
+  for (int i = w; i < k; i += nw) {  // |D_i| and the ascending lists, one warp per row
+    int base = 0;
+    for (int j0 = 0; j0 < d; j0 += 32) {
+      const int j = j0 + lane;
+      const bool on = j < d && dm[i * d + j];
+      const unsigned b = __ballot_sync(0xffffffffu, on);
+      if (on) p.dlist[i * d + base + __popc(b & ((1u << lane) - 1u))] = j;
+      base += __popc(b);
+    }
+    if (lane == 0) T.S->nD[i] = base;
   }
   for (int c = tid; c < kd; c += bd) p.dmask[c] = dm[c];
   __syncthreads();
+  TST(T, 7);
 }
 
 // ------------------------------------------------------------ iteration prologue
 // Medoid rows of MCur (fp64), delta_i (Alg 3 l.4-7, reading R6), and the
 // active slots of GPU-FAST-PROCLUS: new medoids get their Dist row computed,
-// cached ones with a changed radius get the band of Theorem 3.1.
+// cached ones with a changed radius get the band of Theorem 3.1.  With
+// T.mrow the rows of M and the DistFound / delta' tables are read from the
+// shared-memory copies the cost tail loaded up front.
 __device__ void prepare_s(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
-  const int k = p.k, d = p.d;
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+  const int k = p.k, d = p.d, tid = threadIdx.x, bd = blockDim.x;
+  const bool cached = T.mrow != nullptr;
+  for (int e = tid; e < k * d; e += bd) {
     const int i = e / d, j = e - i * d;
-    T.med[e] = (double)p.mrows[(long long)S->mcur[i] * d + j];
+    const long long r = (long long)S->mcur[i] * d + j;
+    T.med[e] = (double)(cached ? T.mrow[r] : p.mrows[r]);
   }
-  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+  for (int i = tid; i < k; i += bd) {
     const int mp = S->mcur[i];
-    T.fnd[i] = p.found[mp];
-    T.fnd[KMAX + i] = p.used[mp];
-    T.fnd[2 * KMAX + i] = p.dprev[mp];
+    T.fnd[i] = cached ? T.fall[mp] : p.found[mp];
+    T.fnd[KMAX + i] = cached ? T.uall[mp] : p.used[mp];
+    T.fnd[2 * KMAX + i] = cached ? T.pall[mp] : p.dprev[mp];
   }
   __syncthreads();
-  if (threadIdx.x < k) {
-    const int i = threadIdx.x;
+  TST(T, 15);
+  for (int e = tid; e < k * k; e += bd) {  // one thread per ordered pair (i, j)
+    const int i = e / k, j = e - i * k;
+    T.dd[e] = (i == j) ? CUDART_INF : full_dist(T.med + i * d, 1, T.med + j * d, d, p.metric);
+  }
+  __syncthreads();
+  if (tid < k) {
     double m = CUDART_INF;
     for (int j = 0; j < k; ++j) {
-      if (j == i) continue;
-      const double t = full_dist(T.med + i * d, 1, T.med + j * d, d, p.metric);
+      const double t = T.dd[tid * k + j];
       if (t < m) m = t;
     }
-    S->delta[i] = m;
+    S->delta[tid] = m;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int na = 0;
-    for (int i = 0; i < k; ++i) {
+  TST(T, 16);
+  if (tid < 32) {  // active slots in slot order, one lane per slot
+    const int i = tid;
+    ActSlot a;
+    bool on = false;
+    if (i < k) {
       const double dl = S->delta[i];
       const double dp = T.fnd[2 * KMAX + i];
-      ActSlot a;
       a.slot = i;
       a.mpos = S->mcur[i];
       a.compute = T.fnd[i] != 0.0 ? 0 : 1;
       a.lam = 1;
+      on = true;
       if (T.fnd[KMAX + i] == 0.0) {
         a.lo = -CUDART_INF;
         a.hi = dl;
@@ -864,18 +1463,22 @@ __device__ void prepare_s(const RunParams& p, TailMem& T) {
         a.hi = dp;
         a.lam = -1;
       } else {
-        continue;  // delta unchanged: Delta L_i is empty (eq 3)
+        on = false;  // delta unchanged: Delta L_i is empty (eq 3)
       }
-      S->act[na++] = a;
     }
-    S->n_act = na;
+    const unsigned b = __ballot_sync(0xffffffffu, on);
+    if (on) S->act[__popc(b & ((1u << i) - 1u))] = a;
+    if (i == 0) S->n_act = __popc(b);
   }
   __syncthreads();
+  TST(T, 17);
 }
 
 __global__ void k_prepare(RunParams p) {
   extern __shared__ __align__(16) unsigned char smraw[];
   TailMem T = tail_mem(p, smraw);
+  T.mrow = nullptr;  // first iteration: read M and the tables from global memory
+  TST_START();
   state_load(p, T.S);
   prepare_s(p, T);
   state_store(p, T.S);
@@ -888,127 +1491,203 @@ void launch_prepare(const RunParams& p, cudaStream_t s) {
 // ------------------------------------------------------------ per-pass tails
 // Locality tail: H and |L| updates of Theorem 3.2 / eq 6 and P:203 (in fixed
 // point, so the incremental H is exact integer arithmetic), DistFound /
-// delta' bookkeeping, X = H / |L| and FindDimensions.
+// delta' bookkeeping, X = H / |L| and FindDimensions.  Round trip 1:
+// the state; round trip 2: band sums and counts of every slot (unused ones
+// are zero), the H rows and |L| of MCur, and 2^-e_j.
 __device__ void tail_locality(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
-  const int d = p.d, k = p.k, na = S->n_act;
-  if (threadIdx.x == 0 && na > 0)  // byte model: data once + one Dist row per slot
+  const int d = p.d, k = p.k, kd = k * d, tid = threadIdx.x, bd = blockDim.x;
+  __shared__ long long cnt_s[KMAX], nL_s[KMAX];
+  long long* Hs = (long long*)T.dev;  // [k][d] H rows of MCur by slot
+  long long* va = (long long*)T.Z;    // [na][d] band sums by active slot
+  state_load(p, S);
+  const int na = S->n_act;
+  for (int c = tid; c < kd; c += bd) {
+    const int i = c / d, j = c - i * d;
+    const long long h = __ldcg(p.Hq + (long long)S->mcur[i] * d + j);
+    const long long v = c < na * d ? take_acc(p, c) : 0ll;
+    Hs[c] = h;
+    va[c] = v;
+  }
+  if (tid < k) {
+    const long long nl = __ldcg(p.nL + S->mcur[tid]);
+    const long long v = tid < na ? take_cnt(p, tid) : 0ll;
+    nL_s[tid] = nl;
+    cnt_s[tid] = v;
+  }
+  for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
+  if (tid == 0 && na > 0)  // byte model: data once + one Dist row per slot
     S->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
-  for (int c = threadIdx.x; c < na * d; c += blockDim.x) {
+  __syncthreads();
+  TST(T, 0);
+  for (int c = tid; c < na * d; c += bd) {
     const int a = c / d, j = c - a * d;
     const ActSlot& A = S->act[a];
-    const long long v = take_acc(p, c);
-    p.Hq[(long long)A.mpos * d + j] += (A.lam > 0 ? v : -v);
+    const int e = A.slot * d + j;
+    const long long h = Hs[e] + (A.lam > 0 ? va[c] : -va[c]);
+    Hs[e] = h;
+    p.Hq[(long long)A.mpos * d + j] = h;
   }
-  if (threadIdx.x < na) {
-    const ActSlot& A = S->act[threadIdx.x];
-    const long long v = take_cnt(p, threadIdx.x);
-    p.nL[A.mpos] += (A.lam > 0 ? v : -v);
+  if (tid < na) {
+    const ActSlot& A = S->act[tid];
+    const long long nl = nL_s[A.slot] + (A.lam > 0 ? cnt_s[tid] : -cnt_s[tid]);
+    nL_s[A.slot] = nl;
+    p.nL[A.mpos] = nl;
     p.dprev[A.mpos] = S->delta[A.slot];
     p.used[A.mpos] = 1;
     p.found[A.mpos] = 1;
   }
-  __threadfence_block();
   __syncthreads();
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
+  for (int c = tid; c < kd; c += bd) {
     const int i = c / d, j = c - i * d;
-    const int mp = S->mcur[i];
-    T.X[c] = ddiv(dmul((double)p.Hq[(long long)mp * d + j], p.iscale[j]), (double)p.nL[mp]);
+    T.X[c] = ddiv(dmul((double)Hs[c], T.isc[j]), (double)nL_s[i]);
   }
   __syncthreads();
+  TST(T, 1);
   zscore_select_s(p, T);
   const int it = S->iterations;
   if (p.tr.cap > 0 && it < p.tr.cap) {
-    for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-      if (p.tr.X) p.tr.X[(long long)it * k * d + c] = T.X[c];
-      if (p.tr.dims) p.tr.dims[(long long)it * k * d + c] = T.dm[c];
+    for (int c = tid; c < kd; c += bd) {
+      if (p.tr.X) p.tr.X[(long long)it * kd + c] = T.X[c];
+      if (p.tr.dims) p.tr.dims[(long long)it * kd + c] = T.dm[c];
     }
-    if (threadIdx.x < k) {
-      const int i = threadIdx.x;
-      if (p.tr.mcur) p.tr.mcur[it * k + i] = S->mcur[i];
-      if (p.tr.delta) p.tr.delta[it * k + i] = S->delta[i];
-      if (p.tr.nL) p.tr.nL[it * k + i] = p.nL[S->mcur[i]];
+    if (tid < k) {
+      if (p.tr.mcur) p.tr.mcur[it * k + tid] = S->mcur[tid];
+      if (p.tr.delta) p.tr.delta[it * k + tid] = S->delta[tid];
+      if (p.tr.nL) p.tr.nL[it * k + tid] = nL_s[tid];
     }
   }
 }
 
 // Assign tail: |C_i| and the centroid mu_ij = sum / |C_i| on j in D_i.
+// One round trip: state, sums, counts, dimension lists and 2^-e_j together.
 __device__ void tail_assign(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
-  const int d = p.d, k = p.k;
-  if (threadIdx.x < k) S->sizes[threadIdx.x] = take_cnt(p, threadIdx.x);
-  __syncthreads();
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d, t = c - i * d;
-    const long long sz = S->sizes[i];
+  const int d = p.d, k = p.k, kd = k * d, tid = threadIdx.x, bd = blockDim.x;
+  __shared__ long long sz_s[KMAX];
+  long long* raw = (long long*)T.Z;
+  StateRegs sr;
+  state_issue(p, sr);
+  for (int c = tid; c < kd; c += bd) {
+    const int dl = p.dlist[c];
     const long long v = take_acc(p, c);
+    T.dl[c] = dl;
+    raw[c] = v;
+  }
+  if (tid < k) sz_s[tid] = take_cnt(p, tid);
+  for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
+  state_commit(p, sr, S);
+  __syncthreads();
+  TST(T, 20);
+  if (tid < k) S->sizes[tid] = sz_s[tid];
+  for (int c = tid; c < kd; c += bd) {
+    const int i = c / d, t = c - i * d;
+    const long long sz = sz_s[i];
     double m = 0.0;
-    if (t < S->nD[i] && sz > 0) m = ddiv(dmul((double)v, p.iscale[p.dlist[c]]), (double)sz);
+    if (t < S->nD[i] && sz > 0) m = ddiv(dmul((double)raw[c], T.isc[T.dl[c]]), (double)sz);
     p.mu[c] = m;
   }
+  TST(T, 21);
 }
 
 // Cost tail: eq 1-2 with the |Data| denominator (eq 8, reading R4), then
 // Alg 1 l.10-14: keep the best, ComputeBadMedoids (reading R11),
 // replace bad medoids from M \ MBest (reading R12), stop after itrPat
-// iterations without improvement, and prepare the next iteration.
+// iterations without improvement, and prepare the next iteration.  One round
+// trip brings the state, the deviation sums, the dimension lists, 2^-e_j and
+// (when cached) the rows of M with their DistFound / delta' entries, so the
+// prologue of the next iteration needs no further global loads.
 __device__ void tail_cost(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
-  const int k = p.k, d = p.d;
-  __shared__ unsigned bad_s;
-  __shared__ int np_s;
+  const int k = p.k, d = p.d, kd = k * d, nM = p.nM;
+  const int tid = threadIdx.x, bd = blockDim.x, lane = tid & 31;
   __shared__ double cw_s[KMAX];
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d, t = c - i * d;
+  long long* raw = (long long*)T.Z;
+  StateRegs sr;
+  state_issue(p, sr);
+  for (int c = tid; c < kd; c += bd) {
+    const int dl = p.dlist[c];
     const long long v = take_acc(p, c);
-    T.dev[c] = (t < S->nD[i]) ? dmul((double)v, p.iscale[p.dlist[c]]) : 0.0;
+    T.dl[c] = dl;
+    raw[c] = v;
+  }
+  for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
+  if (T.mrow) {
+    for (int e = tid; e < nM * d; e += bd) T.mrow[e] = p.mrows[e];
+    for (int m = tid; m < nM; m += bd) {
+      T.fall[m] = p.found[m];
+      T.uall[m] = p.used[m];
+      T.pall[m] = p.dprev[m];
+    }
+  }
+  state_commit(p, sr, S);
+  __syncthreads();
+  TST(T, 10);
+  for (int c = tid; c < kd; c += bd) {  // dev_it and the per-term quotients of eq 1
+    const int i = c / d, t = c - i * d;
+    const long long ci = S->sizes[i];
+    const bool on = t < S->nD[i];
+    const double dv = on ? dmul((double)raw[c], T.isc[T.dl[c]]) : 0.0;
+    T.dev[c] = dv;
+    T.Z[c] = (on && ci != 0) ? ddiv(dv, (double)ci) : 0.0;
   }
   __syncthreads();
-  if (threadIdx.x < k) {  // |C_i| * w_i of eq 1, one cluster per thread
-    const int i = threadIdx.x;
+  if (tid < k) {  // |C_i| * w_i of eq 1, terms added in t order
+    const int i = tid;
     const long long c = S->sizes[i];
     double cw = 0.0;
     if (c != 0) {
-      double w = 0.0;
+      double wv = 0.0;
       const int nd = S->nD[i];
-      for (int t = 0; t < nd; ++t) w = dadd(w, ddiv(T.dev[i * d + t], (double)c));
-      w = ddiv(w, (double)nd);
-      cw = dmul((double)c, w);
+      for (int t = 0; t < nd; ++t) wv = dadd(wv, T.Z[i * d + t]);
+      wv = ddiv(wv, (double)nd);
+      cw = dmul((double)c, wv);
     }
     cw_s[i] = cw;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
+  TST(T, 11);
+  if (tid < 32) {  // control, one warp
+    const unsigned full = 0xffffffffu;
     double cost = 0.0;
-    for (int i = 0; i < k; ++i)  // eq 2 / eq 8, i ascending; empty clusters add 0
-      if (S->sizes[i] != 0) cost = dadd(cost, cw_s[i]);
-    cost = ddiv(cost, (double)p.n_total);
-    S->cost = cost;
-    S->itr += 1;
+    if (lane == 0) {
+      for (int i = 0; i < k; ++i)  // eq 2 / eq 8, i ascending; empty clusters add 0
+        if (S->sizes[i] != 0) cost = dadd(cost, cw_s[i]);
+      cost = ddiv(cost, (double)p.n_total);
+    }
+    cost = __shfl_sync(full, cost, 0);
     const int it = S->iterations;
-    S->iterations = it + 1;
     const int improved = cost < S->cost_best;
-    S->improved = improved;
-    if (improved) {
-      S->itr = 0;
-      S->cost_best = cost;
-      for (int i = 0; i < k; ++i) {
-        S->mbest[i] = S->mcur[i];
-        S->sizes_best[i] = S->sizes[i];
+    __syncwarp();
+    if (improved && lane < k) {
+      S->mbest[lane] = S->mcur[lane];
+      S->sizes_best[lane] = S->sizes[lane];
+    }
+    if (lane == 0) {
+      S->cost = cost;
+      S->itr = improved ? 0 : S->itr + 1;
+      S->iterations = it + 1;
+      S->improved = improved;
+      if (improved) {
+        S->cost_best = cost;
+        S->best_buf = S->cur_buf;
+        S->cur_buf ^= 1;
       }
-      S->best_buf = S->cur_buf;
-      S->cur_buf ^= 1;
     }
-    unsigned bad = 0u;
+    __syncwarp();
+    // bad medoids (R11): |C_i| < n/k * minDev in CBest, else the smallest
     const double thr = dmul(ddiv((double)p.n_total, (double)k), p.minDev);
-    int smallest = 0;
-    for (int i = 0; i < k; ++i) {
-      if ((double)S->sizes_best[i] < thr) bad |= 1u << i;
-      if (S->sizes_best[i] < S->sizes_best[smallest]) smallest = i;
+    const long long sb = lane < k ? S->sizes_best[lane] : 0ll;
+    unsigned bad = __ballot_sync(full, lane < k && (double)sb < thr);
+    if (!bad) {  // first smallest |C_i| (sizes are < 2^63, non-negative)
+      const unsigned long long u = lane < k ? (unsigned long long)sb : ~0ull;
+      const unsigned hi = (unsigned)(u >> 32), lo = (unsigned)u;
+      const unsigned mhi = __reduce_min_sync(full, hi);
+      const unsigned mlo = __reduce_min_sync(full, hi == mhi ? lo : 0xffffffffu);
+      const unsigned at = __reduce_min_sync(full, (hi == mhi && lo == mlo) ? (unsigned)lane : 32u);
+      bad = 1u << at;
     }
-    if (!bad) bad = 1u << smallest;
-    bad_s = bad;
-    if (p.tr.cap > 0 && it < p.tr.cap) {
+    if (lane == 0 && p.tr.cap > 0 && it < p.tr.cap) {
       if (p.tr.cost) p.tr.cost[it] = cost;
       if (p.tr.improved) p.tr.improved[it] = (unsigned char)improved;
       for (int i = 0; i < k; ++i) {
@@ -1016,41 +1695,45 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
         if (p.tr.bad) p.tr.bad[it * k + i] = (bad >> i) & 1u;
       }
     }
-    for (int i = 0; i < k; ++i) S->mcur[i] = S->mbest[i];
-  }
-  __syncthreads();
-  if (threadIdx.x < 32) {  // pool = ascending positions of M not in MBest
-    int base = 0;
-    for (int t0 = 0; t0 < p.nM; t0 += 32) {
-      const int t = t0 + threadIdx.x;
-      bool inb = t >= p.nM;
+    if (lane < k) S->mcur[lane] = S->mbest[lane];
+    __syncwarp();
+    // pool = ascending positions of M not in MBest
+    int np = 0;
+    for (int t0 = 0; t0 < nM; t0 += 32) {
+      const int t = t0 + lane;
+      bool inb = t >= nM;
       if (!inb)
         for (int i = 0; i < k; ++i) inb |= (S->mbest[i] == t);
-      const unsigned b = __ballot_sync(0xffffffffu, !inb);
-      if (!inb) T.pool[base + __popc(b & ((1u << threadIdx.x) - 1u))] = t;
-      base += __popc(b);
+      const unsigned b = __ballot_sync(full, !inb);
+      if (!inb) T.pool[np + __popc(b & ((1u << lane) - 1u))] = t;
+      np += __popc(b);
     }
-    if (threadIdx.x == 0) np_s = base;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    // replacement draws (stream IT): the r-th remaining pool entry, in order
-    const unsigned bad = bad_s;
-    int np = np_s;
+    __syncwarp();
+    // replacement draws (stream IT): the r-th remaining pool entry, in order;
+    // every lane runs the same generator, the removal shift is warp-wide
     unsigned long long rng = S->rng;
     for (int i = 0; i < k; ++i) {
       if (!((bad >> i) & 1u) || np == 0) continue;
       const int r = (int)sm64_uniform(&rng, (unsigned long long)np);
-      S->mcur[i] = T.pool[r];
-      for (int t = r; t + 1 < np; ++t) T.pool[t] = T.pool[t + 1];
+      if (lane == 0) S->mcur[i] = T.pool[r];
+      for (int t0 = r; t0 < np - 1; t0 += 32) {
+        const int t = t0 + lane;
+        const int v = t < np - 1 ? T.pool[t + 1] : 0;
+        __syncwarp();
+        if (t < np - 1) T.pool[t] = v;
+        __syncwarp();
+      }
       --np;
     }
-    S->rng = rng;
-    S->done = (S->itr >= p.itrPat || S->iterations >= p.max_iter) ? 1 : 0;
-    if (p.use_cond)
-      cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, S->done ? 0u : 1u);
+    if (lane == 0) {
+      S->rng = rng;
+      S->done = (S->itr >= p.itrPat || S->iterations >= p.max_iter) ? 1 : 0;
+      if (p.use_cond)
+        cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, S->done ? 0u : 1u);
+    }
   }
   __syncthreads();
+  TST(T, 14);
   if (!S->done) prepare_s(p, T);
 }
 
@@ -1059,24 +1742,26 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
 // Delta_i = min_{j != i} seg_{D*_i}(m_i, m_j) (reading R5).
 __device__ void tail_refine(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
-  const int k = p.k, d = p.d;
+  const int k = p.k, d = p.d, kd = k * d, tid = threadIdx.x, bd = blockDim.x;
   __shared__ long long sz_s[KMAX];
-  if (threadIdx.x < k) sz_s[threadIdx.x] = take_cnt(p, threadIdx.x);
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+  long long* raw = (long long*)T.Z;
+  StateRegs sr;
+  state_issue(p, sr);
+  for (int c = tid; c < kd; c += bd) raw[c] = take_acc(p, c);
+  if (tid < k) sz_s[tid] = take_cnt(p, tid);
+  for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
+  state_commit(p, sr, S);
+  __syncthreads();
+  for (int e = tid; e < kd; e += bd) {
     const int i = e / d, j = e - i * d;
     T.med[e] = (double)p.mrows[(long long)S->mbest[i] * d + j];
-  }
-  __syncthreads();
-  for (int c = threadIdx.x; c < k * d; c += blockDim.x) {
-    const int i = c / d, j = c - i * d;
     const long long sz = sz_s[i];
-    const long long v = take_acc(p, c);
-    T.X[c] = sz > 0 ? ddiv(dmul((double)v, p.iscale[j]), (double)sz) : 0.0;
+    T.X[e] = sz > 0 ? ddiv(dmul((double)raw[e], T.isc[j]), (double)sz) : 0.0;
   }
   __syncthreads();
   zscore_select_s(p, T);
-  if (threadIdx.x < k) {
-    const int i = threadIdx.x;
+  if (tid < k) {
+    const int i = tid;
     double m = CUDART_INF;
     for (int j = 0; j < k; ++j) {
       if (j == i) continue;
@@ -1094,14 +1779,16 @@ __device__ void tail_refine(const RunParams& p, TailMem& T) {
   }
 }
 
-// Run a tail: load the state into shared memory, run it, store it back.
+// Run a tail (each tail loads the state itself), store the state back.  The
+// tickets are stored as 0: the copy may predate last_block()'s reset.
 #define RUN_TAIL(FN, KIND)                                          \
   do {                                                              \
     const unsigned long long t0_ = gtimer();                        \
     TailMem T_ = tail_mem(p, smraw + p.lay[LAYK].tail);             \
-    state_load(p, T_.S);                                            \
+    TST_START();                                                    \
     FN(p, T_);                                                      \
     __syncthreads();                                                \
+    if (threadIdx.x < 4) T_.S->ticket[threadIdx.x] = 0u;            \
     if (threadIdx.x == 0) T_.S->tail_ns[KIND] += gtimer() - t0_;    \
     state_store(p, T_.S);                                           \
   } while (0)
@@ -1241,9 +1928,10 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
       const int metric = p.metric;
       long long gp = (long long)blockIdx.x * P + q;
       const long long gstep = (long long)gridDim.x * P;
-      for (long long i = 0; i < nmy; ++i, gp += gstep) {
-        const int stg = (int)(i % p.stages);
-        mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+      RingPos rp;
+      for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
+        const int stg = rp.stg;
+        mbar_wait(&R.full[stg], rp.ph);
         const float* xs = R.buf + (size_t)stg * R.rows * P;
         const bool valid = gp < p.n;
         float xr[DR > 0 ? DR : 1];
@@ -1329,6 +2017,65 @@ struct __align__(8) Term {
 };
 #define LDX(base, boff) (*reinterpret_cast<const float*>(reinterpret_cast<const char*>(base) + (boff)))
 
+// Segmental distance terms of one cluster for PPT points: fp32 partial sums
+// in two chains (the certified bound only needs the number of terms, DESIGN.md
+// section 5).  ND is the compile-time |D_i| (fully unrolled); the _n variant
+// handles |D_i| > 16.
+template <int PPT, int ND>
+__device__ __forceinline__ void dist_terms(const float* __restrict__ xq,
+                                           const Term* __restrict__ tb, float (&s)[PPT]) {
+  float a[PPT], b[PPT];
+#pragma unroll
+  for (int u = 0; u < PPT; ++u) {
+    a[u] = 0.f;
+    b[u] = 0.f;
+  }
+#pragma unroll
+  for (int t = 0; t < ND; t += 2) {
+    const Term e0 = tb[t];
+    if (t + 1 < ND) {
+      const Term e1 = tb[t + 1];
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) {
+        a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
+        b[u] += fabsf(LDX(xq + u * 32, e1.joff) - e1.m);
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < PPT; ++u) s[u] = ND > 1 ? a[u] + b[u] : a[u];
+}
+
+template <int PPT>
+__device__ __noinline__ void dist_terms_n(const float* __restrict__ xq, const Term* __restrict__ tb,
+                                          int nd, float (&s)[PPT]) {
+  float a[PPT], b[PPT];
+#pragma unroll
+  for (int u = 0; u < PPT; ++u) {
+    a[u] = 0.f;
+    b[u] = 0.f;
+  }
+  int t = 0;
+  for (; t + 2 <= nd; t += 2) {
+    const Term e0 = tb[t], e1 = tb[t + 1];
+#pragma unroll
+    for (int u = 0; u < PPT; ++u) {
+      a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
+      b[u] += fabsf(LDX(xq + u * 32, e1.joff) - e1.m);
+    }
+  }
+  if (t < nd) {
+    const Term e = tb[t];
+#pragma unroll
+    for (int u = 0; u < PPT; ++u) a[u] += fabsf(LDX(xq + u * 32, e.joff) - e.m);
+  }
+#pragma unroll
+  for (int u = 0; u < PPT; ++u) s[u] = a[u] + b[u];
+}
+
 template <int PPT>
 __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   DevState* st = p.st;
@@ -1389,9 +2136,10 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     const int q0 = w * 32 * PPT;
     long long base = (long long)blockIdx.x * P;
     const long long gstep = (long long)gridDim.x * P;
-    for (long long i = 0; i < nmy; ++i, base += gstep) {
-      const int stg = (int)(i % p.stages);
-      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      mbar_wait(&R.full[stg], rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const float* xq = xs + q0 + lane;
       float best[PPT], second[PPT];
@@ -1407,41 +2155,22 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         const int nd = nD_s[c];
         // fp32 partial sums in any order: the certified bound only needs the
         // number of terms; 4 terms in flight per point
-        float s[PPT], s2[PPT];
-#pragma unroll
-        for (int u = 0; u < PPT; ++u) {
-          s[u] = 0.f;
-          s2[u] = 0.f;
-        }
-        int t = 0;
-        for (; t + 4 <= nd; t += 4) {
-          const Term e0 = tb[t], e1 = tb[t + 1], e2 = tb[t + 2], e3 = tb[t + 3];
-#pragma unroll
-          for (int u = 0; u < PPT; ++u) {
-            const float* xu = xq + u * 32;
-            s[u] += fabsf(LDX(xu, e0.joff) - e0.m) + fabsf(LDX(xu, e1.joff) - e1.m);
-            s2[u] += fabsf(LDX(xu, e2.joff) - e2.m) + fabsf(LDX(xu, e3.joff) - e3.m);
-          }
-        }
-        if (t + 2 <= nd) {
-          const Term e0 = tb[t], e1 = tb[t + 1];
-#pragma unroll
-          for (int u = 0; u < PPT; ++u) {
-            const float* xu = xq + u * 32;
-            s[u] += fabsf(LDX(xu, e0.joff) - e0.m);
-            s2[u] += fabsf(LDX(xu, e1.joff) - e1.m);
-          }
-          t += 2;
-        }
-        if (t < nd) {
-          const Term e = tb[t];
-#pragma unroll
-          for (int u = 0; u < PPT; ++u) s[u] += fabsf(LDX(xq + u * 32, e.joff) - e.m);
+        float s[PPT];
+        switch (nd) {
+#define DT(N) \
+  case N:     \
+    dist_terms<PPT, N>(xq, tb, s); \
+    break;
+          DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+          DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+#undef DT
+          default:
+            dist_terms_n<PPT>(xq, tb, nd, s);
         }
         const float r = rcp_s[c];
 #pragma unroll
         for (int u = 0; u < PPT; ++u) {
-          const float qv = (s[u] + s2[u]) * r;
+          const float qv = s[u] * r;
           second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);
           bi[u] = qv < best[u] ? c : bi[u];
           best[u] = fminf(best[u], qv);
@@ -1544,9 +2273,10 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
     const int q = w * 32 + lane;
     long long gp = (long long)blockIdx.x * P + q;
     const long long gstep = (long long)gridDim.x * P;
-    for (long long i = 0; i < nmy; ++i, gp += gstep) {
-      const int stg = (int)(i % p.stages);
-      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      mbar_wait(&R.full[stg], rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const int lb = gp < p.n ? (int)R.lab[(size_t)stg * P + q] : -1;
       // one ballot per cluster: lane c of the warp keeps cluster c's mask
@@ -1621,10 +2351,11 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
     pipe_produce(p, R, nmy, nullptr, nullptr);
   } else {
     const int q0 = w * 32 * PPT;
-    for (long long i = 0; i < nmy; ++i) {
-      const int stg = (int)(i % p.stages);
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, rp.next(p.stages)) {
+      const int stg = rp.stg;
       const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
-      mbar_wait(&R.full[stg], (unsigned)((i / p.stages) & 1));
+      mbar_wait(&R.full[stg], rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
 #pragma unroll
       for (int u = 0; u < PPT; ++u) {
@@ -1681,7 +2412,6 @@ __global__ void k_tail(RunParams p, int tail) {
   DevState* st = p.st;
   if (tail != TAIL_REF && st->done) return;
   TailMem T = tail_mem(p, smraw);
-  state_load(p, T.S);
   if (tail == TAIL_LOC)
     tail_locality(p, T);
   else if (tail == TAIL_ASG)
@@ -1730,6 +2460,22 @@ static TailLayout tail_layout(int d, int k, int nM) {
   t.dm = b.take(kd);
   t.pool = b.take(4 * (size_t)(nM > 0 ? nM : 1));
   t.fnd = b.take(8 * 3 * KMAX);
+  t.isc = b.take(8 * (size_t)d);
+  t.dl = b.take(4 * kd);
+  t.dd = b.take(8 * (size_t)k * k);
+  // the cost tail caches M (fp32 rows + DistFound / delta' tables) when small
+  const size_t m = (size_t)(nM > 0 ? nM : 1);
+  LB c = b;
+  const int mrow = c.take(4 * m * d), fall = c.take(m), uall = c.take(m), pall = c.take(8 * m);
+  if (c.off <= 40 * 1024) {
+    b = c;
+    t.mrow = mrow;
+    t.fall = fall;
+    t.uall = uall;
+    t.pall = pall;
+  } else {
+    t.mrow = t.fall = t.uall = t.pall = -1;
+  }
   t.bytes = (int)((b.off + 15) & ~(size_t)15);
   return t;
 }
@@ -1843,18 +2589,36 @@ PassShape pass_shape(int d, int k, int nM, int num_sms) {
   ps.smem_ref = ps.smem_cost;
   ps.smem_fin = ps.lay[KK_FIN].bytes;
   // persistent grids: as many resident blocks per SM as shared memory and
-  // the 2048-thread limit allow (<= 8), per kernel
-  auto grid_of = [&](size_t smem, int tpb) {
-    int per_sm = (int)((227 * 1024) / (smem + 1024));
+  // the 2048-thread limit and the register file allow (<= 8), per kernel, so
+  // that the whole grid is one resident wave
+  auto grid_of = [&](const void* fn, size_t smem, int tpb) {
+    cudaFuncAttributes fa;
+    size_t stat = 0;
+    int regs = 0;
+    if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) {
+      stat = fa.sharedSizeBytes;
+      regs = fa.numRegs;
+    } else {
+      cudaGetLastError();
+    }
+    int per_sm = (int)((227 * 1024) / (smem + stat + 1024));
     if (per_sm > 2048 / tpb) per_sm = 2048 / tpb;
+    if (regs > 0) {
+      const int warp_regs = ((regs * 32 + 255) / 256) * 256;
+      const int by_regs = 65536 / (warp_regs * ((tpb + 31) / 32));
+      if (per_sm > by_regs) per_sm = by_regs;
+    }
     if (per_sm > 8) per_sm = 8;
     if (per_sm < 1) per_sm = 1;
     return num_sms * per_sm;
   };
-  ps.grid_loc = grid_of(ps.smem_loc, ps.tpb_loc);
-  ps.grid_asg = grid_of(ps.smem_asg, ps.tpb_asg);
-  ps.grid_lsum = grid_of(ps.smem_cost, ps.tpb_lsum);
-  ps.grid_fin = grid_of(ps.smem_fin, ps.tpb_fin);
+  const void* loc_fn = d <= 16 ? (const void*)k_locality<16>
+                       : d <= 32 ? (const void*)k_locality<32>
+                                 : (const void*)k_locality<0>;
+  ps.grid_loc = grid_of(loc_fn, ps.smem_loc, ps.tpb_loc);
+  ps.grid_asg = grid_of((const void*)k_assign<2>, ps.smem_asg, ps.tpb_asg);
+  ps.grid_lsum = grid_of((const void*)k_labelsum<0>, ps.smem_cost, ps.tpb_lsum);
+  ps.grid_fin = grid_of((const void*)k_final<2>, ps.smem_fin, ps.tpb_fin);
   ps.grid = ps.grid_loc;
   ps.per_sm = ps.grid_loc / num_sms;
   return ps;
