@@ -255,6 +255,9 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
     if (m > 0.f) {
       const double bound = 2.0 * (double)h->n_total * (double)m;
       e = 61 - (int)std::ceil(std::log2(bound));
+      // one term (<= 2 max|x_j|) stays below 2^51: the per-term quantisation
+      // of the lane-private passes keeps it in the low mantissa bits of a double
+      e = std::min(e, 50 - (int)std::ceil(std::log2(2.0 * (double)m)));
       e = std::max(-1000, std::min(1000, e));
     }
     sc[(size_t)j] = std::ldexp(1.0, e);
@@ -592,7 +595,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
                                   uint64_t seed, proclus_result* out) {
   const int d = h->d;
   const int nM = (int)h->nM;
-  const PassShape ps = pass_shape(d, k, nM, h->num_sms);
+  const PassShape ps = pass_shape(d, k, l, nM, h->num_sms);
   CK(configure_kernels(ps));
   CK(h->lab.ensure((size_t)2 * h->n_pad));
   CK(h->med.ensure((size_t)KMAX * d));
@@ -677,7 +680,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.st = h->st.p;
   p.P = ps.P;
   p.stages = ps.stages;
-  for (int q = 0; q < 4; ++q) p.lay[q] = ps.lay[q];
+  for (int q = 0; q < NLAY; ++q) p.lay[q] = ps.lay[q];
   p.tl = ps.tl;
   p.tail_smem = ps.tail_smem;
   p.nchunks = (h->n + ps.P - 1) / ps.P;

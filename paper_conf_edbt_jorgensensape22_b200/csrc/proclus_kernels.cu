@@ -789,6 +789,37 @@ __device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+// Per-warp phase cycle counters (-DPROCLUS_PHASE_PROFILE builds only):
+// PH_MARK(i) adds the cycles since the previous mark to phase i (i < 0:
+// restart); PH_FLUSH adds them (lane 0 of each warp, iteration 3 only) to
+// dbg_cyc[base + i] and the number of warps to dbg_cyc[base + 4].
+#ifdef PROCLUS_PHASE_PROFILE
+#define PH_DECL()                      \
+  unsigned long long ph_t[4] = {0, 0, 0, 0}; \
+  unsigned long long ph_last = clock64()
+#define PH_MARK(i)                                   \
+  do {                                               \
+    const unsigned long long ph_now = clock64();     \
+    if ((i) >= 0) ph_t[(i) < 0 ? 0 : (i)] += ph_now - ph_last; \
+    ph_last = ph_now;                                \
+  } while (0)
+#define PH_FLUSH(ST, BASE)                                                    \
+  do {                                                                        \
+    if ((threadIdx.x & 31) == 0 && (ST)->iterations == 3) {                   \
+      for (int ph_i = 0; ph_i < 4; ++ph_i) atomicAdd(&(ST)->dbg_cyc[(BASE) + ph_i], ph_t[ph_i]); \
+      atomicAdd(&(ST)->dbg_cyc[(BASE) + 4], 1ull);                            \
+    }                                                                         \
+  } while (0)
+#else
+#define PH_DECL() do {} while (0)
+#define PH_MARK(i) do {} while (0)
+#define PH_FLUSH(ST, BASE) do {} while (0)
+#endif
+
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -2305,6 +2336,720 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
 #undef LAYK
 }
 
+// ============================================================ lane-private sums
+// Per-term fixed point: the term t (|x - c| or x) of dimension j becomes
+// round(t * 2^e_j) as an int64 via the 1.5 * 2^52 "magic" addend -- one DFMA
+// forms x*2^e_j - c*2^e_j (c*2^e_j exact: a power-of-two scale) with one
+// rounding, one DADD rounds it to an integer held in the low mantissa bits
+// (|t| 2^e_j < 2^51 by the choice of e_j, proclus_api.cu).  The int64 values
+// are added exactly, so the totals do not depend on the order, the grid or the
+// number of GPUs; the error per term is <= 2^-(e_j+1).
+constexpr double QMAGIC_D = 6755399441055744.0;  // 1.5 * 2^52
+constexpr long long QMAGIC_BITS = 0x4338000000000000ll;
+__device__ __forceinline__ long long q_abs(float x, double sc, double cq) {
+  const double r = __fma_rn((double)x, sc, -cq);
+  return __double_as_longlong(__dadd_rn(fabs(r), QMAGIC_D)) - QMAGIC_BITS;
+}
+__device__ __forceinline__ long long q_val(float x, double sc) {
+  return __double_as_longlong(__fma_rn((double)x, sc, QMAGIC_D)) - QMAGIC_BITS;
+}
+
+// Producer of the kernels with their own chunk geometry (SmemLayout P, ldr,
+// stages): chunk c covers points [c P, c P + P) clipped to n_pad (a multiple of
+// 32, so every copy stays a multiple of 16 bytes); dimension row j of stage s
+// lands at buf + (s d + j) ldr floats, the labels (if any) at lab + s P.
+__device__ void pipe_produce_k(const RunParams& p, const Pipe& R, const SmemLayout& L,
+                               long long nmy, const unsigned char* labsrc) {
+  const int lane = threadIdx.x & 31;
+  const int P = L.P, d = p.d;
+  int stg = 0, round = 0;
+  for (long long i = 0; i < nmy; ++i) {
+    if (round > 0) {
+      mbar_wait(&R.empty[stg], (unsigned)((round - 1) & 1));
+      fence_proxy_async();
+    }
+    const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
+    const long long left = p.n_pad - base;
+    const unsigned cnt = (unsigned)(left < P ? left : P);
+    const unsigned bytes = cnt * 4u * (unsigned)d + (labsrc ? cnt : 0u);
+    if (lane == 0) mbar_expect_tx(&R.full[stg], bytes);
+    __syncwarp();
+    float* dst = R.buf + (size_t)stg * d * L.ldr;
+    for (int j = lane; j < d; j += 32)
+      bulk_g2s(dst + (size_t)j * L.ldr, p.xs + (size_t)j * p.n_pad + base, cnt * 4u, &R.full[stg]);
+    if (labsrc && lane == 0) bulk_g2s(R.lab + (size_t)stg * P, labsrc + base, cnt, &R.full[stg]);
+    if (++stg == L.stages) {
+      stg = 0;
+      ++round;
+    }
+  }
+}
+__device__ __forceinline__ long long chunks_of_block_k(const RunParams& p, int P) {
+  const long long nch = (p.n + P - 1) / P;
+  return (nch > blockIdx.x) ? (nch - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+}
+
+// One work item of a sorted-member pass: cell (i, t) of dimension j (row
+// offset joff in a ring stage), the residue r of the members it takes
+// (members r, r + R, r + 2R, ... of cluster i in each chunk), 2^e_j and
+// centre * 2^e_j.  Items live in registers-free shared tables; their int64
+// partial sums in an item-private shared array (no two threads share one).
+struct __align__(16) Item {
+  int joff, c, r, R;
+  double sc, cq;
+};
+
+// Counting sort of one chunk's points by cluster (labels in the ring) among
+// the consumer threads: list[base_c + pos] = q for the points of cluster c,
+// hist[c] = |members|, base_s[c] = base_c.  Two named barriers; hist, base
+// and list are double-buffered by chunk parity (hist_next, the other
+// buffer's histogram, is cleared between the two barriers).  The order
+// inside a cluster depends on atomics, which is harmless: every sum over the
+// members is an exact integer sum.
+__device__ __forceinline__ void sort_chunk(const unsigned char* lab_s, long long nvalid, int q,
+                                           int nct, int k, int* hist, int* hist_next, int* base_s,
+                                           int* list) {
+  const int lane = threadIdx.x & 31;
+  const bool valid = q < nvalid;
+  const int c = valid ? (int)lab_s[q] : 0;
+  int pos = 0;
+  if (valid) pos = atomicAdd(&hist[c], 1);
+  named_bar_sync(1, nct);
+  const int h = lane < k ? hist[lane] : 0;
+  int x = h;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  const int base = __shfl_sync(0xffffffffu, x - h, c);
+  if (valid) list[base + pos] = q;
+  if (threadIdx.x < 32 && lane < k) base_s[lane] = x - h;
+  if (threadIdx.x < KMAX) hist_next[threadIdx.x] = 0;  // read last in the previous chunk
+  named_bar_sync(1, nct);
+}
+
+// The same with PPTS points per thread, given as (q[r], c[r]) in registers
+// (c < 0: no point).
+template <int PPTS>
+__device__ __forceinline__ void sort_chunk_m(const int (&q)[PPTS], const int (&c)[PPTS], int nct,
+                                             int k, int* hist, int* hist_next, int* base_s,
+                                             int* list) {
+  const int lane = threadIdx.x & 31;
+  int pos[PPTS];
+#pragma unroll
+  for (int r = 0; r < PPTS; ++r) pos[r] = c[r] >= 0 ? atomicAdd(&hist[c[r]], 1) : 0;
+  named_bar_sync(1, nct);
+  const int h = lane < k ? hist[lane] : 0;
+  int x = h;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+#pragma unroll
+  for (int r = 0; r < PPTS; ++r) {
+    const int base = __shfl_sync(0xffffffffu, x - h, c[r] < 0 ? 0 : c[r]);
+    if (c[r] >= 0) list[base + pos[r]] = q[r];
+  }
+  if (threadIdx.x < 32 && lane < k) base_s[lane] = x - h;
+  if (threadIdx.x < KMAX) hist_next[threadIdx.x] = 0;
+  named_bar_sync(1, nct);
+}
+
+// packed fp32x2 arithmetic (sm_100 FADD2): two points per instruction
+__device__ __forceinline__ float2 f2_sub_abs_add(float2 acc, float2 x, float m) {
+  // acc + |x - m| on both halves (FADD2 with a broadcast operand and |.|)
+  unsigned long long r, a = *reinterpret_cast<unsigned long long*>(&acc),
+                        xv = *reinterpret_cast<unsigned long long*>(&x);
+  unsigned long long mm = ((unsigned long long)__float_as_uint(m) << 32) | __float_as_uint(m);
+  unsigned long long t;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(t) : "l"(xv), "l"(mm));
+  const float2 tf = *reinterpret_cast<float2*>(&t);
+  const float2 ab = make_float2(fabsf(tf.x), fabsf(tf.y));
+  const unsigned long long abv = *reinterpret_cast<const unsigned long long*>(&ab);
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(abv));
+  return *reinterpret_cast<float2*>(&r);
+}
+
+// Per-block state of the sorted-member item machinery (shared memory).
+struct ItemCtx {
+  Item* items;       // [nitem]
+  long long* iacc;   // [nitem] item-private int64 sums
+  int* gix;          // [cells] global cell index i * d + t
+  int* hist0;        // [2][KMAX] histograms + [2][KMAX] bases (double buffer)
+  int* list0;        // [2][P] sorted chunk points
+  long long* ccnt;   // [KMAX] |members| per cluster (MODE 1, 2)
+  int* off_s;        // [KMAX] first cell of cluster i
+  int* nd_s;         // [KMAX] cells of cluster i
+  int* rr_s;         // [KMAX] R_i
+  int* ib_s;         // [KMAX + 1] first item of cluster i
+  int nitem, nct;
+};
+
+// MODE 0: cells (i, t < |D_i|) of |x_j - mu_ij| (cost, Alg 6 l.9-13);
+// MODE 1: cells (i, j < d) of |x_j - mbest_ij| (refinement X, Alg 1 l.16);
+// MODE 2: cells (i, t < |D_i|) of x_j (centroid sums, Alg 6 l.1-8).
+// R_i (threads per cell of cluster i) is proportional to the expected
+// |C_i| (sizes of the current / best / previous clustering).  Block-wide.
+template <int MODE>
+__device__ void items_build(const RunParams& p, const SmemLayout& L, ItemCtx& X) {
+  const DevState* st = p.st;
+  const int d = p.d, k = p.k, lane = threadIdx.x & 31;
+  if (threadIdx.x < 32) {
+    const int i = lane;
+    const int nd = i < k ? (MODE == 1 ? d : st->nD[i]) : 0;
+    const long long sz = i < k ? (MODE == 1 ? st->sizes_best[i] : st->sizes[i]) : 0;
+    int x = nd;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    double wsum = (double)nd * (double)sz;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) wsum += __shfl_xor_sync(0xffffffffu, wsum, o);
+    const int tot = __shfl_sync(0xffffffffu, x, 31);  // number of cells
+    int Ri = 1;
+    if (wsum > 0.0 && i < k) {
+      const double f = floor((double)X.nct * (double)sz / wsum);
+      Ri = f < 1.0 ? 1 : (f > 4096.0 ? 4096 : (int)f);
+    } else if (i < k) {  // no estimate: spread evenly
+      Ri = tot > 0 ? max(1, X.nct / tot) : 1;
+    }
+    const int ni = i < k ? nd * Ri : 0;
+    int y2 = ni;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, y2, o);
+      if (lane >= o) y2 += y;
+    }
+    if (i < k) {
+      X.off_s[i] = x - nd;
+      X.nd_s[i] = nd;
+      X.rr_s[i] = Ri;
+      X.ib_s[i] = y2 - ni;
+    }
+    if (lane == 31) X.ib_s[KMAX] = y2;
+    X.hist0[lane] = 0;
+    X.hist0[KMAX + lane] = 0;
+    if (MODE != 0) X.ccnt[lane] = 0;
+  }
+  __syncthreads();
+  X.nitem = X.ib_s[KMAX];
+  for (int it = threadIdx.x; it < X.nitem; it += blockDim.x) {
+    int i = 0;
+    while (i + 1 < k && X.ib_s[i + 1] <= it) ++i;
+    const int loc = it - X.ib_s[i], nd = X.nd_s[i];
+    const int r = loc / nd, t = loc - r * nd;
+    const int e = i * d + t;
+    const int j = MODE == 1 ? t : p.dlist[e];
+    const double sc = p.scale[j];
+    double c = 0.0;
+    if (MODE == 0) c = p.mu[e];
+    if (MODE == 1) c = (double)p.mrows[(long long)st->mbest[i] * d + j];
+    X.items[it] = Item{j * L.ldr * 4, i, r, X.rr_s[i], sc, c * sc};
+    X.iacc[it] = 0;
+    if (r == 0) X.gix[X.off_s[i] + t] = e;
+  }
+}
+
+// The items of one sorted chunk (after sort_chunk): thread q adds its items'
+// members in registers, then once into its item-private accumulators.
+template <int MODE>
+__device__ __forceinline__ void items_chunk(const ItemCtx& X, const char* xs, const int* hist,
+                                            const int* base_s, const int* list, int q, int k) {
+  for (int it = q; it < X.nitem; it += X.nct) {
+    const Item I = X.items[it];
+    const int cnt = hist[I.c];
+    const int* lm = list + base_s[I.c];
+    const char* xj = xs + I.joff;
+    long long a = 0, b = 0;
+    int m = I.r;
+    // 4 members in flight: their list entries and coordinates are loaded
+    // before any of them is converted
+    for (; m + 3 * I.R < cnt; m += 4 * I.R) {
+      const int q0 = lm[m], q1 = lm[m + I.R], q2 = lm[m + 2 * I.R], q3 = lm[m + 3 * I.R];
+      const float x0 = *reinterpret_cast<const float*>(xj + q0 * 4);
+      const float x1 = *reinterpret_cast<const float*>(xj + q1 * 4);
+      const float x2 = *reinterpret_cast<const float*>(xj + q2 * 4);
+      const float x3 = *reinterpret_cast<const float*>(xj + q3 * 4);
+      if (MODE == 2) {
+        a += q_val(x0, I.sc) + q_val(x1, I.sc);
+        b += q_val(x2, I.sc) + q_val(x3, I.sc);
+      } else {
+        a += q_abs(x0, I.sc, I.cq) + q_abs(x1, I.sc, I.cq);
+        b += q_abs(x2, I.sc, I.cq) + q_abs(x3, I.sc, I.cq);
+      }
+    }
+    for (; m < cnt; m += I.R) {
+      const float x = *reinterpret_cast<const float*>(xj + lm[m] * 4);
+      a += MODE == 2 ? q_val(x, I.sc) : q_abs(x, I.sc, I.cq);
+    }
+    X.iacc[it] += a + b;
+  }
+  if (MODE != 0 && q < k) X.ccnt[q] += hist[q];
+}
+
+// Per cell: the sum of its R_i items; one int64 atomic per cell (and count)
+// per block into one of the NCOPY global copies.  Block-wide.
+template <int MODE>
+__device__ void items_flush(const RunParams& p, const ItemCtx& X) {
+  const int k = p.k;
+  const int cp = blockIdx.x % NCOPY;
+  long long* acc = p.accg + (size_t)cp * p.k * p.d;
+  const int ncell = X.off_s[k - 1] + X.nd_s[k - 1];
+  for (int cell = threadIdx.x; cell < ncell; cell += blockDim.x) {
+    int i = 0;
+    while (i + 1 < k && X.off_s[i + 1] <= cell) ++i;
+    const int t = cell - X.off_s[i], nd = X.nd_s[i];
+    long long s = 0;
+    for (int r = 0; r < X.rr_s[i]; ++r) s += X.iacc[X.ib_s[i] + r * nd + t];
+    if (s) atomicAdd((unsigned long long*)&acc[X.gix[cell]], (unsigned long long)s);
+  }
+  if (MODE != 0) {
+    long long* cnt = p.cntg + (size_t)cp * KMAX;
+    if (threadIdx.x < k && X.ccnt[threadIdx.x])
+      atomicAdd((unsigned long long*)&cnt[threadIdx.x], (unsigned long long)X.ccnt[threadIdx.x]);
+  }
+}
+
+__device__ __forceinline__ ItemCtx item_ctx(const SmemLayout& L, unsigned char* smraw, int* off_s,
+                                            int* nd_s, int* rr_s, int* ib_s) {
+  ItemCtx X;
+  X.items = SMP(Item, tab);
+  X.iacc = SMP(long long, acc);
+  X.gix = SMP(int, nD);
+  X.hist0 = SMP(int, bal);
+  X.list0 = SMP(int, row);
+  X.ccnt = SMP(long long, cnt);
+  X.off_s = off_s;
+  X.nd_s = nd_s;
+  X.rr_s = rr_s;
+  X.ib_s = ib_s;
+  X.nct = L.nw * 32;
+  X.nitem = 0;
+  return X;
+}
+
+__device__ __forceinline__ void pipe_init_k(const SmemLayout& L, const Pipe& R) {
+  if (threadIdx.x == 0) {
+    for (int s2 = 0; s2 < L.stages; ++s2) {
+      mbar_init(&R.full[s2], 1);
+      mbar_init(&R.empty[s2], (unsigned)L.nw);
+    }
+    fence_mbar_init();
+  }
+}
+
+// --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) / refinement X over
+// CBest (Alg 1 l.16-17).  Each chunk is counting-sorted by cluster; every
+// consumer thread owns a fixed set of work items (cell, residue r, stride
+// R_i) for the whole launch, with R_i proportional to the cluster's size, so
+// the members of cluster i are spread evenly over the R_i * |D_i| threads of
+// its cells and each thread adds ~|members| / R_i exact int64 terms per chunk
+// in a register (no shared-memory read-modify-write per term, no walk over
+// ballot masks, no divergence from unequal |D_i|).
+// REF = 0: cells (i, t < |D_i|) of |x_j - mu_ij|; REF = 1: cells (i, j < d)
+// of |x_j - mbest_ij| plus |C_i|.
+template <int REF>
+__global__ void __launch_bounds__(416) k_lsum2(RunParams p) {
+  DevState* st = p.st;
+  if (!REF && st->done) return;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[REF ? KK_REF2 : KK_LS2];
+  const int P = L.P, d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nct = nw * 32;
+  Pipe R = pipe_of(L, smraw, d);
+  __shared__ int off_s[KMAX], nd_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
+  ItemCtx X = item_ctx(L, smraw, off_s, nd_s, rr_s, ib_s);
+  const unsigned char* lab =
+      REF ? (st->best_buf ? p.lab1 : p.lab0) : (st->cur_buf ? p.lab1 : p.lab0);
+  const long long nmy = chunks_of_block_k(p, P);
+  pipe_init_k(L, R);
+  items_build<REF ? 1 : 0>(p, L, X);
+  __syncthreads();
+  if (w == nw) {
+    pipe_produce_k(p, R, L, nmy, lab);
+  } else {
+    const int q = w * 32 + lane;
+    long long g0 = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+    for (long long ch = 0; ch < nmy; ++ch, g0 += gstep, rp.next(L.stages)) {
+      const int stg = rp.stg;
+      const int hb = (int)(ch & 1);
+      int* hist = X.hist0 + hb * KMAX;
+      int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
+      int* list = X.list0 + hb * P;
+      mbar_wait(&R.full[stg], rp.ph);
+      sort_chunk(R.lab + (size_t)stg * P, p.n - g0, q, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX,
+                 base_s, list);
+      items_chunk<REF ? 1 : 0>(X, reinterpret_cast<const char*>(R.buf + (size_t)stg * d * L.ldr),
+                               hist, base_s, list, q, k);
+      pipe_release(R, stg);
+    }
+  }
+  __syncthreads();
+  items_flush<REF ? 1 : 0>(p, X);
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[REF ? 3 : 2])) return;
+  if (REF) {
+#define LAYK KK_REF2
+    RUN_TAIL(tail_refine, 3);
+#undef LAYK
+  } else {
+#define LAYK KK_LS2
+    RUN_TAIL(tail_cost, 2);
+#undef LAYK
+  }
+}
+
+// --- AssignPoints (Alg 5) + centroid sums (Alg 6 l.1-8), d <= 16: every
+// lane holds the 16 coordinates of 2 point PAIRS in registers (LDS.64 once
+// per pair and dimension) and evaluates seg_{D_c} for all clusters with
+// packed fp32x2 adds (FADD2 with |.|); the medoid rows come from shared
+// memory as warp-broadcast float4s and D_c as a bitmask, so a chunk costs
+// 16 coordinate loads per point instead of one gather per (point, term).
+// Certified fp32 argmin + fp64 fallback (reading R8) as in k_assign; then the
+// chunk is counting-sorted by the new labels and the item threads add the
+// centroid terms.  4 consumer warps x 128 points.
+__global__ void __launch_bounds__(160) k_assign3(RunParams p) {
+#ifdef PROCLUS_PHASE_PROFILE
+  const unsigned long long phs = gtimer();
+#endif
+  DevState* st = p.st;
+  if (st->done) return;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_ASG3];
+  const int P = L.P, d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nct = nw * 32;
+  Pipe R = pipe_of(L, smraw, d);
+  __shared__ int off_s[KMAX], nd_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
+  __shared__ float rcp_s[KMAX];
+  __shared__ unsigned msk_s[KMAX];
+  __shared__ int ndmax_s;
+  ItemCtx X = item_ctx(L, smraw, off_s, nd_s, rr_s, ib_s);
+  float* med_s = SMP(float, med);    // [k][16] fp32 rows, zero padded
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nDa);
+  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  const long long nmy = chunks_of_block_k(p, P);
+  pipe_init_k(L, R);
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    const int nd = st->nD[i];
+    nD_s[i] = nd;
+    rcp_s[i] = 1.0f / (float)nd;
+    unsigned m = 0;
+    for (int t = 0; t < nd; ++t) m |= 1u << p.dlist[i * d + t];
+    msk_s[i] = m;
+  }
+  for (int e = threadIdx.x; e < k * 16; e += blockDim.x) {
+    const int i = e >> 4, j = e & 15;
+    med_s[e] = j < d ? p.mrows[(long long)st->mcur[i] * d + j] : 0.f;
+  }
+  for (int e = threadIdx.x; e < k * 16; e += blockDim.x) {
+    const int i = e >> 4, t = e & 15;
+    dl_s[e] = t < d ? p.dlist[i * d + t] : 0;  // stride 16, as med_s
+  }
+  items_build<2>(p, L, X);
+  if (threadIdx.x == 0) {
+    int m = 0;
+    for (int i = 0; i < k; ++i) m = max(m, (int)st->nD[i]);
+    ndmax_s = m;
+  }
+  __syncthreads();
+  const double G = (double)(ndmax_s + 6) * 5.9604644775390625e-08;
+  long long nfb = 0;
+#ifdef PROCLUS_PHASE_PROFILE
+  const unsigned long long ph0 = gtimer();
+#endif
+  if (w == nw) {
+    pipe_produce_k(p, R, L, nmy, nullptr);
+  } else {
+    const int tid = w * 32 + lane;
+    const int q0 = w * 128 + 2 * lane;  // pairs (q0, q0+1) and (q0+64, q0+65)
+    long long g0 = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+    PH_DECL();
+    for (long long ch = 0; ch < nmy; ++ch, g0 += gstep, rp.next(L.stages)) {
+      PH_MARK(-1);
+      const int stg = rp.stg;
+      const int hb = (int)(ch & 1);
+      int* hist = X.hist0 + hb * KMAX;
+      int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
+      int* list = X.list0 + hb * P;
+      mbar_wait(&R.full[stg], rp.ph);
+      PH_MARK(0);
+      const float* xs = R.buf + (size_t)stg * d * L.ldr;
+      float2 xr[16][2];
+#pragma unroll
+      for (int j = 0; j < 16; ++j)
+#pragma unroll
+        for (int u = 0; u < 2; ++u)
+          xr[j][u] = j < d ? *reinterpret_cast<const float2*>(xs + j * L.ldr + q0 + 64 * u)
+                           : make_float2(0.f, 0.f);
+      float best[4], second[4];
+      int bi[4];
+#pragma unroll
+      for (int v = 0; v < 4; ++v) {
+        best[v] = CUDART_INF_F;
+        second[v] = CUDART_INF_F;
+        bi[v] = 0;
+      }
+      for (int c = 0; c < k; ++c) {
+        const unsigned msk = msk_s[c];
+        const float4* m4 = reinterpret_cast<const float4*>(med_s + c * 16);
+        float2 s0 = make_float2(0.f, 0.f), s1 = s0;
+        // D_c nibble by nibble: one warp-uniform jump per 4 dimensions into a
+        // case that applies exactly the selected dimensions (no predicated
+        // work for the dimensions outside D_c)
+#define NIB_CASE(N, J4)                                                        \
+  case N:                                                                      \
+    if ((N)&1) { s0 = f2_sub_abs_add(s0, xr[4 * J4][0], mv.x); s1 = f2_sub_abs_add(s1, xr[4 * J4][1], mv.x); } \
+    if ((N)&2) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 1][0], mv.y); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 1][1], mv.y); } \
+    if ((N)&4) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 2][0], mv.z); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 2][1], mv.z); } \
+    if ((N)&8) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 3][0], mv.w); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 3][1], mv.w); } \
+    break;
+#define NIB_SWITCH(J4)                                                         \
+  {                                                                            \
+    const unsigned nib = (msk >> (4 * J4)) & 15u;                              \
+    if (nib) {                                                                 \
+      const float4 mv = m4[J4];                                                \
+      switch (nib) {                                                           \
+        NIB_CASE(1, J4) NIB_CASE(2, J4) NIB_CASE(3, J4) NIB_CASE(4, J4)        \
+        NIB_CASE(5, J4) NIB_CASE(6, J4) NIB_CASE(7, J4) NIB_CASE(8, J4)        \
+        NIB_CASE(9, J4) NIB_CASE(10, J4) NIB_CASE(11, J4) NIB_CASE(12, J4)     \
+        NIB_CASE(13, J4) NIB_CASE(14, J4) NIB_CASE(15, J4)                     \
+        default: break;                                                        \
+      }                                                                        \
+    }                                                                          \
+  }
+        NIB_SWITCH(0) NIB_SWITCH(1) NIB_SWITCH(2) NIB_SWITCH(3)
+#undef NIB_SWITCH
+#undef NIB_CASE
+        const float r = rcp_s[c];
+        const float qv[4] = {s0.x * r, s0.y * r, s1.x * r, s1.y * r};
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+          second[v] = qv[v] < best[v] ? best[v] : fminf(second[v], qv[v]);
+          bi[v] = qv[v] < best[v] ? c : bi[v];
+          best[v] = fminf(best[v], qv[v]);
+        }
+      }
+      int qv4[4], cv4[4];
+#pragma unroll
+      for (int v = 0; v < 4; ++v) {
+        const int q = q0 + (v >> 1) * 64 + (v & 1);
+        const long long gp = g0 + q;
+        int lbl = bi[v];
+        if (gp < p.n) {
+          const bool certain = (best[v] >= 1e-30f) && (second[v] < 1e30f) &&
+                               ((double)second[v] * (1.0 - G) > (double)best[v] * (1.0 + G));
+          if (!certain) {
+            lbl = exact_argmin(xs + q, L.ldr, med_s, dl_s, nD_s, k, 16, nullptr, nullptr);
+            ++nfb;
+          }
+        }
+        qv4[v] = q;
+        cv4[v] = gp < p.n ? lbl : -1;
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int q = q0 + 64 * u;
+        const unsigned short two =
+            (unsigned short)((cv4[2 * u] & 0xff) | ((cv4[2 * u + 1] & 0xff) << 8));
+        if (g0 + q + 1 < p.n) {
+          *reinterpret_cast<unsigned short*>(lab + g0 + q) = two;
+        } else if (g0 + q < p.n) {
+          lab[g0 + q] = (unsigned char)cv4[2 * u];
+        }
+      }
+      PH_MARK(1);
+      sort_chunk_m<4>(qv4, cv4, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX, base_s, list);
+      PH_MARK(2);
+      items_chunk<2>(X, reinterpret_cast<const char*>(xs), hist, base_s, list, tid, k);
+      PH_MARK(3);
+      pipe_release(R, stg);
+    }
+    PH_FLUSH(st, 10);
+  }
+#ifdef PROCLUS_PHASE_PROFILE
+  const unsigned long long ph1 = gtimer();
+#endif
+  __syncthreads();
+  items_flush<2>(p, X);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
+#ifdef PROCLUS_PHASE_PROFILE
+  __syncthreads();
+  if (threadIdx.x == 0 && st->iterations == 3) {
+    const unsigned long long ph2 = gtimer();
+    atomicAdd(&st->dbg_cyc[4], ph0 - phs);
+    atomicAdd(&st->dbg_cyc[5], ph1 - ph0);
+    atomicAdd(&st->dbg_cyc[6], ph2 - ph1);
+    atomicAdd(&st->dbg_cyc[7], 1ull);
+    atomicMax(&st->dbg_cyc[8], ~phs);
+    atomicMax(&st->dbg_cyc[9], ph2);
+  }
+#endif
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[1])) return;
+#define LAYK KK_ASG3
+  RUN_TAIL(tail_assign, 1);
+#undef LAYK
+}
+
+// --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8)
+// on sorted chunks: (1) one thread per point takes the certified fp32
+// argmin of seg_{D_i}(x, m_i) (fp64 fallback near a tie, reading R8) and
+// writes its u8 label; (2) the chunk is counting-sorted by the new labels;
+// (3) the item threads add the centroid terms x_j, j in D_i, exactly.
+__global__ void __launch_bounds__(416) k_assign2(RunParams p) {
+  DevState* st = p.st;
+  if (st->done) return;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_ASG2];
+  const int P = L.P, d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nct = nw * 32;
+  Pipe R = pipe_of(L, smraw, d);
+  __shared__ int off_s[KMAX], nd_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
+  __shared__ float rcp_s[KMAX];
+  __shared__ int ndmax_s;
+  ItemCtx X = item_ctx(L, smraw, off_s, nd_s, rr_s, ib_s);
+  float* med_s = SMP(float, med);
+  Term* tab_s = SMP(Term, tab2);
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nDa);
+  unsigned char* labq = SMP(unsigned char, labq);  // [P] this chunk's labels
+  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  const long long nmy = chunks_of_block_k(p, P);
+  pipe_init_k(L, R);
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    const int nd = st->nD[i];
+    nD_s[i] = nd;
+    rcp_s[i] = 1.0f / (float)nd;
+  }
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
+    dl_s[e] = p.dlist[e];
+  }
+  items_build<2>(p, L, X);
+  __syncthreads();
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i]) {
+      const int j = dl_s[e];
+      tab_s[e].joff = j * L.ldr * 4;
+      tab_s[e].m = med_s[i * d + j];
+    }
+  }
+  if (threadIdx.x == 0) {
+    int m = 0;
+    for (int i = 0; i < k; ++i) m = max(m, nD_s[i]);
+    ndmax_s = m;
+  }
+  __syncthreads();
+  const double G = (double)(ndmax_s + 6) * 5.9604644775390625e-08;
+  long long nfb = 0;
+  if (w == nw) {
+    pipe_produce_k(p, R, L, nmy, nullptr);
+  } else {
+    const int q = w * 32 + lane;
+    long long g0 = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+#ifdef PROCLUS_PHASE_PROFILE
+    unsigned long long tw = 0, tdd = 0, tso = 0, tit = 0;
+#endif
+    for (long long ch = 0; ch < nmy; ++ch, g0 += gstep, rp.next(L.stages)) {
+      const int stg = rp.stg;
+      const int hb = (int)(ch & 1);
+      int* hist = X.hist0 + hb * KMAX;
+      int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
+      int* list = X.list0 + hb * P;
+#ifdef PROCLUS_PHASE_PROFILE
+      const unsigned long long c0 = clock64();
+#endif
+      mbar_wait(&R.full[stg], rp.ph);
+#ifdef PROCLUS_PHASE_PROFILE
+      const unsigned long long c1 = clock64();
+      tw += c1 - c0;
+#endif
+      const float* xs = R.buf + (size_t)stg * d * L.ldr;
+      const long long gp = g0 + q;
+      if (gp < p.n) {
+        const float* xq = xs + q;
+        float best = CUDART_INF_F, second = CUDART_INF_F;
+        int bi = 0;
+        const Term* tb = tab_s;
+        for (int c = 0; c < k; ++c, tb += d) {
+          float sv[1];
+          switch (nD_s[c]) {
+#define DT(N) \
+  case N:     \
+    dist_terms<1, N>(xq, tb, sv); \
+    break;
+            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+#undef DT
+            default:
+              dist_terms_n<1>(xq, tb, nD_s[c], sv);
+          }
+          const float qv = sv[0] * rcp_s[c];
+          second = qv < best ? best : fminf(second, qv);
+          bi = qv < best ? c : bi;
+          best = fminf(best, qv);
+        }
+        const bool certain = (best >= 1e-30f) && (second < 1e30f) &&
+                             ((double)second * (1.0 - G) > (double)best * (1.0 + G));
+        int lbl = bi;
+        if (!certain) {
+          lbl = exact_argmin(xq, L.ldr, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
+          ++nfb;
+        }
+        lab[gp] = (unsigned char)lbl;
+        labq[q] = (unsigned char)lbl;
+      }
+#ifdef PROCLUS_PHASE_PROFILE
+      const unsigned long long c2 = clock64();
+      tdd += c2 - c1;
+#endif
+      sort_chunk(labq, p.n - g0, q, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX, base_s, list);
+#ifdef PROCLUS_PHASE_PROFILE
+      const unsigned long long c3 = clock64();
+      tso += c3 - c2;
+#endif
+      items_chunk<2>(X, reinterpret_cast<const char*>(xs), hist, base_s, list, q, k);
+#ifdef PROCLUS_PHASE_PROFILE
+      tit += clock64() - c3;
+#endif
+      pipe_release(R, stg);
+    }
+#ifdef PROCLUS_PHASE_PROFILE
+    if (lane == 0 && st->iterations == 3) {
+      atomicAdd(&st->dbg_cyc[10], tw);
+      atomicAdd(&st->dbg_cyc[11], tdd);
+      atomicAdd(&st->dbg_cyc[12], tso);
+      atomicAdd(&st->dbg_cyc[13], tit);
+      atomicAdd(&st->dbg_cyc[14], 1ull);
+    }
+#endif
+  }
+  __syncthreads();
+  items_flush<2>(p, X);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[1])) return;
+#define LAYK KK_ASG2
+  RUN_TAIL(tail_assign, 1);
+#undef LAYK
+}
+
 // --- Final AssignPoints with D* (Alg 1 l.18) and RemoveOutliers (l.19):
 // outlier iff seg_{D*_i}(x, m_i) > Delta_i for every i (reading R17).
 template <int PPT>
@@ -2487,7 +3232,7 @@ static void finish(SmemLayout& L, LB& b, const TailLayout& tl) {
   L.bytes = (int)((end + 64 + 15) & ~(size_t)15);
 }
 
-PassShape pass_shape(int d, int k, int nM, int num_sms) {
+PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   PassShape ps;
   int P = 256, stages = 3;
   const int cfg[6][2] = {{256, 3}, {256, 2}, {128, 3}, {128, 2}, {64, 3}, {64, 2}};
@@ -2583,6 +3328,93 @@ PassShape pass_shape(int d, int k, int nM, int num_sms) {
     finish(L, b, ps.tl);
     ps.lay[KK_FIN] = L;
   }
+  // lane-private accumulator passes (k_lsum2): the most consumer warps whose
+  // accumulators [nw][cells][32] int64 fit next to the ring
+  // sorted-member passes (k_lsum2): 12 consumer warps, chunks of 384 points,
+  // ring rows padded by 4 floats (conflict-free row gathers)
+  auto ls2_layout = [&](int ncell, bool asg, int& nw_out) -> SmemLayout {
+    SmemLayout best = blank_layout();
+    nw_out = 0;
+    for (int nw = 12; nw >= 4; nw -= 4) {
+      for (int stg = 3; stg >= 2; --stg) {
+        const int Pk = 32 * nw;
+        const int imax = 32 * nw + ncell;  // sum_i |D_i| R_i <= lanes + cells
+        SmemLayout L = blank_layout();
+        LB b;
+        L.nw = nw;
+        L.P = Pk;
+        L.ldr = Pk + 4;
+        L.stages = stg;
+        L.full = b.take(8 * SMAX);
+        L.empty = b.take(8 * SMAX);
+        L.buf = b.take((size_t)stg * d * (Pk + 4) * 4);
+        L.lab = b.take((size_t)stg * Pk);
+        L.tab = b.take(sizeof(Item) * (size_t)imax);
+        L.acc = b.take(8 * (size_t)imax);
+        L.nD = b.take(4 * kd);
+        L.bal = b.take(4 * 4 * KMAX);
+        L.row = b.take(4 * 2 * (size_t)Pk);
+        L.cnt = b.take(8 * KMAX);
+        if (asg) {
+          L.lab = -1;
+          L.med = b.take(4 * kd);
+          L.tab2 = b.take(sizeof(Term) * kd);
+          L.dl = b.take(4 * kd);
+          L.nDa = b.take(4 * KMAX);
+          L.labq = b.take((size_t)Pk);
+        }
+        finish(L, b, ps.tl);
+        if (L.bytes <= 110 * 1024) {
+          nw_out = nw;
+          return L;
+        }
+      }
+    }
+    return best;
+  };
+  {
+    int nw = 0;
+    ps.lay[KK_LS2] = ls2_layout(k * l, false, nw);  // the cost cells: sum |D_i| = k*l
+    ps.lsum2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
+    ps.tpb_ls2 = 32 * (nw + 1);
+    ps.smem_ls2 = ps.lsum2 ? ps.lay[KK_LS2].bytes : 0;
+    ps.lay[KK_REF2] = ls2_layout((int)kd, false, nw);
+    ps.ref2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
+    ps.tpb_ref2 = 32 * (nw + 1);
+    ps.smem_ref2 = ps.ref2 ? ps.lay[KK_REF2].bytes : 0;
+    {  // k_assign3: 4 consumer warps x 128 points, d <= 16
+      SmemLayout L = blank_layout();
+      LB b;
+      const int nw3 = 4, Pk = 512, stg = 3;
+      const int imax = 32 * nw3 + k * l;
+      L.nw = nw3;
+      L.P = Pk;
+      L.ldr = Pk + 4;
+      L.stages = stg;
+      L.full = b.take(8 * SMAX);
+      L.empty = b.take(8 * SMAX);
+      L.buf = b.take((size_t)stg * d * (Pk + 4) * 4);
+      L.tab = b.take(sizeof(Item) * (size_t)imax);
+      L.acc = b.take(8 * (size_t)imax);
+      L.nD = b.take(4 * kd);
+      L.bal = b.take(4 * 4 * KMAX);
+      L.row = b.take(4 * 2 * (size_t)Pk);
+      L.cnt = b.take(8 * KMAX);
+      L.med = b.take(4 * 16 * (size_t)k);
+      L.dl = b.take(4 * 16 * (size_t)k);
+      L.nDa = b.take(4 * KMAX);
+      L.labq = b.take((size_t)Pk);
+      finish(L, b, ps.tl);
+      ps.lay[KK_ASG3] = L;
+      ps.asg3 = d <= 16 && L.bytes <= 113 * 1024 && getenv("PROCLUS_ASSIGN3");
+      ps.tpb_asg3 = 32 * (nw3 + 1);
+      ps.smem_asg3 = ps.asg3 ? L.bytes : 0;
+    }
+    ps.lay[KK_ASG2] = ls2_layout(k * l, true, nw);
+    ps.asg2 = nw >= 4 && getenv("PROCLUS_ASSIGN2");
+    ps.tpb_asg2 = 32 * (nw + 1);
+    ps.smem_asg2 = ps.asg2 ? ps.lay[KK_ASG2].bytes : 0;
+  }
   ps.smem_loc = ps.lay[KK_LOC].bytes;
   ps.smem_asg = ps.lay[KK_ASG].bytes;
   ps.smem_cost = ps.lay[KK_LSUM].bytes;
@@ -2619,6 +3451,10 @@ PassShape pass_shape(int d, int k, int nM, int num_sms) {
   ps.grid_asg = grid_of((const void*)k_assign<2>, ps.smem_asg, ps.tpb_asg);
   ps.grid_lsum = grid_of((const void*)k_labelsum<0>, ps.smem_cost, ps.tpb_lsum);
   ps.grid_fin = grid_of((const void*)k_final<2>, ps.smem_fin, ps.tpb_fin);
+  ps.grid_ls2 = ps.lsum2 ? grid_of((const void*)k_lsum2<0>, ps.smem_ls2, ps.tpb_ls2) : 0;
+  ps.grid_ref2 = ps.ref2 ? grid_of((const void*)k_lsum2<1>, ps.smem_ref2, ps.tpb_ref2) : 0;
+  ps.grid_asg2 = ps.asg2 ? grid_of((const void*)k_assign2, ps.smem_asg2, ps.tpb_asg2) : 0;
+  ps.grid_asg3 = ps.asg3 ? grid_of((const void*)k_assign3, ps.smem_asg3, ps.tpb_asg3) : 0;
   ps.grid = ps.grid_loc;
   ps.per_sm = ps.grid_loc / num_sms;
   return ps;
@@ -2637,6 +3473,26 @@ cudaError_t configure_kernels(const PassShape& ps) {
     e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm[i]);
     if (e != cudaSuccess) return e;
   }
+  if (ps.lsum2) {
+    e = cudaFuncSetAttribute((const void*)k_lsum2<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ps.smem_ls2);
+    if (e != cudaSuccess) return e;
+  }
+  if (ps.ref2) {
+    e = cudaFuncSetAttribute((const void*)k_lsum2<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ps.smem_ref2);
+    if (e != cudaSuccess) return e;
+  }
+  if (ps.asg2) {
+    e = cudaFuncSetAttribute((const void*)k_assign2, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ps.smem_asg2);
+    if (e != cudaSuccess) return e;
+  }
+  if (ps.asg3) {
+    e = cudaFuncSetAttribute((const void*)k_assign3, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ps.smem_asg3);
+    if (e != cudaSuccess) return e;
+  }
   return cudaSuccess;
 }
 
@@ -2649,13 +3505,24 @@ void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  if (ps.asg3)
+    k_assign3<<<ps.grid_asg3, ps.tpb_asg3, ps.smem_asg3, s>>>(p);
+  else if (ps.asg2)
+    k_assign2<<<ps.grid_asg2, ps.tpb_asg2, ps.smem_asg2, s>>>(p);
+  else
+    k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_labelsum<0><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_cost, s>>>(p);
+  if (ps.lsum2)
+    k_lsum2<0><<<ps.grid_ls2, ps.tpb_ls2, ps.smem_ls2, s>>>(p);
+  else
+    k_labelsum<0><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_cost, s>>>(p);
 }
 void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_labelsum<1><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_ref, s>>>(p);
+  if (ps.ref2)
+    k_lsum2<1><<<ps.grid_ref2, ps.tpb_ref2, ps.smem_ref2, s>>>(p);
+  else
+    k_labelsum<1><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_ref, s>>>(p);
 }
 void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s) {
   k_final<2><<<ps.grid_fin, ps.tpb_fin, ps.smem_fin, s>>>(p);

@@ -17,7 +17,14 @@ struct PassShape {
   int grid;       // persistent blocks (SM count x per_sm)
   int grid_loc, grid_asg, grid_lsum, grid_fin;  // per kernel
   size_t smem_loc, smem_asg, smem_cost, smem_ref, smem_fin;
-  SmemLayout lay[4];  // per KernelKind
+  SmemLayout lay[NLAY];  // per KernelKind
+  int lsum2, ref2;       // 1: lane-private accumulator passes (k_lsum2) fit in shared memory
+  int asg2;              // 1: sorted-member assign pass (k_assign2)
+  int asg3;              // 1: register-resident assign pass (k_assign3, d <= 16)
+  int grid_asg3, tpb_asg3;
+  size_t smem_asg3;
+  int grid_ls2, grid_ref2, grid_asg2, tpb_ls2, tpb_ref2, tpb_asg2;
+  size_t smem_ls2, smem_ref2, smem_asg2;
   TailLayout tl;
   int tail_smem;
 };
@@ -40,7 +47,7 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
 void launch_gather_m(const float* srows, const long long* sids, const int* spos, int nM, int d,
                      float* mrows, long long* mids, cudaStream_t s);
 
-PassShape pass_shape(int d, int k, int nM, int num_sms);
+PassShape pass_shape(int d, int k, int l, int nM, int num_sms);
 cudaError_t configure_kernels(const PassShape& ps);
 
 // iteration prologue (delta, active slots) for the state's MCur

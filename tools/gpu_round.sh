@@ -3,8 +3,8 @@
 set -u
 TAG=${1:-x}
 OUT=gpurun_out/$TAG; mkdir -p $OUT
-timeout 400 python -m pytest tests/test_gpu_parity.py -q -x > $OUT/tests.log 2>&1; tail -3 $OUT/tests.log
-timeout 300 python bench.py --steps 20 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/bench.json 2> $OUT/bench.err
+timeout 300 python -m pytest tests/test_gpu_parity.py -q -x > $OUT/tests.log 2>&1; tail -3 $OUT/tests.log
+timeout 200 python bench.py --steps 20 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/bench.json 2> $OUT/bench.err
 python - "$OUT/bench.json" <<'PY'
 import json, sys
 j = json.loads(open(sys.argv[1]).read().strip().splitlines()[-1])
