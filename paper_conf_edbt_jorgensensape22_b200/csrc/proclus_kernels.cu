@@ -837,6 +837,7 @@ struct Pipe {
   unsigned long long* full;   // [SMAX]
   unsigned long long* empty;  // [SMAX]
   int rows;
+  int ldr;                    // row stride in floats (>= P)
 };
 
 __device__ __forceinline__ void pipe_init(const RunParams& p, const Pipe& R, int nw) {
@@ -865,10 +866,10 @@ __device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
     const long long base = (blockIdx.x + i * gridDim.x) * (long long)p.P;
     if (lane == 0) mbar_expect_tx(&R.full[stg], bytes);
     __syncwarp();
-    float* dst = R.buf + (size_t)stg * R.rows * p.P;
+    float* dst = R.buf + (size_t)stg * R.rows * R.ldr;
     for (int j = lane; j < p.d + nex; j += 32) {
       const float* src = j < p.d ? p.xs + (size_t)j * p.n_pad + base : ex->src[j - p.d] + base;
-      bulk_g2s(dst + (size_t)j * p.P, src, row, &R.full[stg]);
+      bulk_g2s(dst + (size_t)j * R.ldr, src, row, &R.full[stg]);
     }
     if (labsrc && lane == 0)
       bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, &R.full[stg]);
@@ -1040,6 +1041,7 @@ struct CarveSize {
 __device__ Pipe carve_pipe(Carve& cv, const RunParams& p, int rows, bool with_lab) {
   Pipe R;
   R.rows = rows;
+  R.ldr = p.P;
   R.full = cv.take<unsigned long long>(SMAX);
   R.empty = cv.take<unsigned long long>(SMAX);
   R.buf = cv.take<float>((size_t)p.stages * rows * p.P);
@@ -1841,6 +1843,7 @@ __device__ __forceinline__ Pipe pipe_of(const SmemLayout& L, unsigned char* smra
   R.buf = SMP(float, buf);
   R.lab = L.lab >= 0 ? SMP(unsigned char, lab) : nullptr;
   R.rows = rows;
+  R.ldr = L.ldr > 0 ? L.ldr : L.P;
   return R;
 }
 
@@ -1892,6 +1895,49 @@ __device__ __forceinline__ Thr make_thr(double lo, double hi, double G) {
   return t;
 }
 
+// Band sums of eq 6 for d <= 16, one lane per (half-warp h, dimension j):
+// both half-warps walk the same member mask of slot a (half h takes the
+// members at even / odd positions), so every lane of the warp does the same
+// number of visits whatever the band sizes (the lane-per-cell walk of
+// warp_cells is as slow as its largest cell).  Each visit reads one point's
+// d coordinates across the lanes of a half (rows padded to LD = P + 4: at
+// most 2-way bank conflicts).  fp64 sums of the exact fp64 terms
+// |x_j - m_aj|, combined over the two halves, quantised to int64 at 2^e_j
+// per (slot, dimension, 32-point sub-chunk) exactly as warp_cells does.
+__device__ __forceinline__ void band_sums_d16(const float* __restrict__ xs, int LD, int q0,
+                                              const float* __restrict__ med_s, int MS, int na,
+                                              int d, const unsigned* __restrict__ bal,
+                                              long long* __restrict__ acc,
+                                              const double* __restrict__ scale_s) {
+  const int lane = threadIdx.x & 31, h = lane >> 4, j = lane & 15;
+  const bool jv = j < d;
+  const float* xr = xs + (size_t)(jv ? j : 0) * LD + q0;
+  const double sc = scale_s[jv ? j : 0];
+  for (int a = 0; a < na; ++a) {
+    unsigned m = bal[a];
+    if (h) m &= m - 1u;  // half 1 starts at the second member
+    const double c = (double)med_s[a * MS + (jv ? j : 0)];
+    double s0 = 0.0, s1 = 0.0;
+    while (m) {
+      const int b0 = __ffs(m) - 1;
+      m &= m - 1u;
+      m &= m - 1u;
+      const float x0 = xr[b0];
+      if (m) {
+        const int b1 = __ffs(m) - 1;
+        m &= m - 1u;
+        m &= m - 1u;
+        const float x1 = xr[b1];
+        s1 = dadd(s1, fabs(dsub((double)x1, c)));
+      }
+      s0 = dadd(s0, fabs(dsub((double)x0, c)));
+    }
+    double s = dadd(s0, s1);
+    s = dadd(s, __shfl_xor_sync(0xffffffffu, s, 16));
+    if (h == 0 && jv && s != 0.0) acc[a * d + j] += __double2ll_rn(dmul(s, sc));
+  }
+}
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
 // One point per lane; the cached Dist rows of the active slots arrive through
 // the same TMA ring as the data (rows d..).  DR: coordinates in registers.
@@ -1907,6 +1953,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   const int na = st->n_act;
   const int ncap = k * d;
   const Pipe R = pipe_of(L, smraw, d + k);
+  const int LD = R.ldr;
   float* med_s = SMP(float, med);
   ActSlot* act_s = SMP(ActSlot, act);
   int* row_s = SMP(int, row);
@@ -1934,7 +1981,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
     const bool cached = a < na && !act_s[a].compute;
     const unsigned b = __ballot_sync(0xffffffffu, cached);
     const int r = __popc(b & ((1u << a) - 1u));
-    if (a < na) row_s[a] = cached ? (d + r) * P : -1;
+    if (a < na) row_s[a] = cached ? (d + r) * R.ldr : -1;
     if (cached) ex->src[r] = p.dist + (size_t)act_s[a].mpos * p.n_pad;
     if (a == 0) ex->n = __popc(b);
   }
@@ -1963,12 +2010,12 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
       for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
         const int stg = rp.stg;
         mbar_wait(&R.full[stg], rp.ph);
-        const float* xs = R.buf + (size_t)stg * R.rows * P;
+        const float* xs = R.buf + (size_t)stg * R.rows * LD;
         const bool valid = gp < p.n;
         float xr[DR > 0 ? DR : 1];
         if (DR > 0) {
 #pragma unroll
-          for (int j = 0; j < DR; ++j) xr[j] = (j < d) ? xs[j * P + q] : 0.f;
+          for (int j = 0; j < DR; ++j) xr[j] = (j < d) ? xs[j * LD + q] : 0.f;
         }
         for (int a = 0; a < na; ++a) {
           const int rs = row_s[a];
@@ -2002,7 +2049,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
                   s = sqrtf(s + s1);
                 }
               } else {
-                s = approx_full(xs + q, P, m, d, metric);
+                s = approx_full(xs + q, LD, m, d, metric);
               }
               f = s;
               p.dist[(long long)act_s[a].mpos * p.n_pad + gp] = f;
@@ -2016,7 +2063,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
               in = false;
             } else {  // within the fp32 error bound: the oracle's fp64 value
               const ActSlot A = act_s[a];
-              const double dv = full_dist(xs + q, P, med_s + a * MS, d, metric);
+              const double dv = full_dist(xs + q, LD, med_s + a * MS, d, metric);
               in = (dv > A.lo) && (dv <= A.hi);
               ++nfb;
             }
@@ -2026,7 +2073,10 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
         __syncwarp();
         if (lane < na) cnt_s[w * KMAX + lane] += __popc(bal[lane]);
         // cells (a, j): band sum of |x_j - m_aj| (eq 6)
-        warp_cells<1, 1>(xs, P, w * 32, cells, na * d, bal, acc, scale_s);
+        if (DR == 16)
+          band_sums_d16(xs, LD, w * 32, med_s, MS, na, d, bal, acc, scale_s);
+        else
+          warp_cells<1, 1>(xs, LD, w * 32, cells, na * d, bal, acc, scale_s);
         pipe_release(R, stg);
       }
     }
@@ -3255,9 +3305,13 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     SmemLayout L = blank_layout();
     LB b;
     L.nw = nw1;
+    L.P = P;
+    // d <= 16: rows padded by 4 floats so that the lane-per-dimension band
+    // sums of k_locality read a point's d coordinates from distinct banks
+    L.ldr = d <= 16 ? P + 4 : P;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
-    L.buf = b.take((size_t)stages * (d + k) * P * 4);
+    L.buf = b.take((size_t)stages * (d + k) * L.ldr * 4);
     L.med = b.take(4 * (size_t)k * (d < 32 ? 32 : d));  // rows padded to 16 / 32
     L.act = b.take(sizeof(ActSlot) * KMAX);
     L.row = b.take(4 * KMAX);
@@ -3275,6 +3329,8 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     SmemLayout L = blank_layout();
     LB b;
     L.nw = nw2;
+    L.P = P;
+    L.ldr = P;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
     L.buf = b.take((size_t)stages * d * P * 4);
@@ -3296,6 +3352,8 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     SmemLayout L = blank_layout();
     LB b;
     L.nw = nw1;
+    L.P = P;
+    L.ldr = P;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
     L.buf = b.take((size_t)stages * d * P * 4);
@@ -3316,6 +3374,8 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     SmemLayout L = blank_layout();
     LB b;
     L.nw = nw2;
+    L.P = P;
+    L.ldr = P;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
     L.buf = b.take((size_t)stages * d * P * 4);
