@@ -145,7 +145,9 @@ def run_reference(args):
     if rank != 0:
         return 0
     oracle.build()
-    data, cfg = synth.config_data(args.config, seed=args.data_seed)
+    # C5 (the sweep) is timed on its data (C3's) one setting per step
+    data, cfg = synth.config_data("C3" if args.config == "C5" else args.config,
+                                  seed=args.data_seed)
     ns = min(REF_SAMPLE_ROWS, cfg["n"])
     sample = np.ascontiguousarray(data[:ns])
     metric = 0 if args.metric == "l2" else 1
@@ -362,13 +364,134 @@ def run_gpu(args):
     return 0
 
 
+SWEEP_KS = list(range(5, 21))   # C5: k in {5..20}
+SWEEP_LS = list(range(3, 11))   # C5: l in {3..10}
+
+
+def run_sweep(args):
+    """--config C5: the multi-parameter sweep of
+    BASELINE.json configs[4] -- k in {5..20} x l in {3..10} (128 settings) at
+    n=1M, d=15 through proclus_run_multi with reuse level 2 (S and M drawn
+    once for k_max; Dist rows, H, delta', |L| shared by every setting).  One
+    step = one whole sweep; value = settings (clusterings) per second.  The
+    same 128 settings as independent proclus_run calls are timed beside it
+    (the paper's level-0 baseline of Fig 3e)."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_edbt_jorgensensape22_b200 as pk
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} needs torchrun with {args.gpus} processes")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    pk.lib()
+    data, cfg = synth.config_data("C3", seed=args.data_seed)  # same 1M x 15 data as C3
+    n, d = cfg["n"], cfg["d"]
+    metric = pk.METRIC_L2 if args.metric == "l2" else pk.METRIC_L1
+    from paper_conf_edbt_jorgensensape22_b200.sharding import shard_rows
+
+    lo, hi = shard_rows(n, world, rank)
+    shard = np.ascontiguousarray(data[lo:hi])
+    uid = None
+    if world > 1:
+        obj = [torch.cuda.nccl.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    stream = torch.cuda.Stream()
+    xdev = torch.from_numpy(shard).cuda()
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device="cuda")
+    h = pk.Proclus(xdev, metric=metric, device=local, stream=stream.cuda_stream,
+                   world_size=world, rank=rank, n_global=n if world > 1 else 0,
+                   row_offset=lo if world > 1 else 0, nccl_unique_id=uid)
+    nset = len(SWEEP_KS) * len(SWEEP_LS)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+        torch.cuda.synchronize()
+
+    def timed(fn, steps):
+        out = []
+        for s in range(steps):
+            with torch.cuda.stream(stream):
+                flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            fn(s)
+            e1.record(stream)
+            e1.synchronize()
+            out.append(e0.elapsed_time(e1))
+        return out
+
+    sweep = lambda s: h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + s, reuse_level=2)
+    for s in range(args.warmup):
+        h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + 1000 + s, reuse_level=2)
+    barrier()
+    with ClockSampler(local) as clk:
+        barrier()
+        ms = timed(sweep, args.steps)
+        barrier()
+    total_ms = sum(ms)
+    # level 0: the same settings as independent runs (one step)
+    indep = lambda s: [h.run(k, l, seed=args.seed0 + s) for k in SWEEP_KS for l in SWEEP_LS]
+    ms0 = timed(indep, 1)
+    ms1 = timed(lambda s: h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + s, reuse_level=1), 1)
+    if world > 1:
+        t = torch.tensor([total_ms, ms0[0], ms1[0]], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms, ms0[0], ms1[0] = (float(v) for v in t.tolist())
+    value = args.steps * nset / (total_ms / 1e3)
+    cpu = None
+    if world == 1 and rank == 0 and not args.no_cpu_baseline:
+        import oracle
+
+        oracle.build()
+        ns = REF_SAMPLE_ROWS
+        ks, ls = [SWEEP_KS[0], SWEEP_KS[-1]], [SWEEP_LS[0], SWEEP_LS[-1]]
+        t0 = time.perf_counter()
+        oracle.proclus_multi(np.ascontiguousarray(data[:ns]), ks, ls, seed=1, reuse_level=2,
+                             metric=0 if args.metric == "l2" else 1)
+        dt = (time.perf_counter() - t0) * n / ns
+        cpu = {"value": len(ks) * len(ls) / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"oracle multi-parameter run (level 2) of the corner settings "
+                         f"k in {ks} x l in {ls} on the first {ns:,} rows, scaled by n/n_sample"}
+    h.close()
+    if rank == 0:
+        line = {
+            "metric": BASELINE_METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": total_ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"C5: multi-parameter sweep k in 5..20 x l in 3..10 "
+                                   f"({nset} settings) at n={n:,} d={d}, reuse level 2 "
+                                   f"(P:207-213), A=100 B=10 minDev=0.7 itrPat=5",
+                       "settings_per_step": nset, "l2": "256 MiB L2 flush between steps",
+                       "parallelism": f"rows sharded over {world} GPU(s)" if world > 1 else "1 GPU"},
+            "sweep_ms": {"level2": total_ms / args.steps, "level1": ms1[0],
+                         "independent_runs": ms0[0]},
+            "reuse_speedup": {"level1": ms0[0] / ms1[0], "level2": ms0[0] / (total_ms / args.steps)},
+            "cpu_baseline": cpu, "clocks": clk.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier(device_ids=[local])
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", choices=["C1", "C2", "C3", "C4"], default="C3")
+    ap.add_argument("--config", choices=["C1", "C2", "C3", "C4", "C5"], default="C3")
     ap.add_argument("--metric", choices=["l2", "l1"], default="l2")
     ap.add_argument("--data-seed", type=int, default=1)
     ap.add_argument("--seed0", type=int, default=1)
@@ -379,6 +502,8 @@ def main():
         args.warmup = 3  # timing rule: at least 3 warm-up steps
     if args.impl == "reference":
         return run_reference(args)
+    if args.config == "C5":
+        return run_sweep(args)
     return run_gpu(args)
 
 

@@ -1258,10 +1258,10 @@ __device__ __forceinline__ int warp_argmin_row(const unsigned long long* keys, i
 // selection of Alg 4 l.15-16 (reading R10): per medoid the two smallest by
 // (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j).  The order is
 // taken on order-preserving 64-bit keys of Z (T.dev); the rest is selected by
-// rank (each free cell counts the free cells before it) when k*d <= 2048,
-// else by a block-wide radix select.  Writes D as a mask (T.dm), |D_i|
+// sorted warp lists (k*d <= 32 * warps), a rank scan (k*d <= 512), else a
+// block-wide radix select (8 passes of 8-bit histograms).  Writes D as a mask (T.dm), |D_i|
 // (S->nD) and, in global memory, the mask and the ascending dimension lists
-// used by the passes.  Needs X in T.X; clobbers T.Z and T.dev.
+// used by the passes.  Needs X in T.X; clobbers T.Z and T.dev (keys / sorted lists).
 __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   __shared__ double Ys[KMAX], Ss[KMAX];
   const int tid = threadIdx.x, bd = blockDim.x, lane = tid & 31, w = tid >> 5, nw = bd >> 5;
@@ -1304,18 +1304,124 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   }
   __syncthreads();
   TST(T, 3);
-  for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
-    const int j1 = warp_argmin_row(key + i * d, d, -1);
-    const int j2 = warp_argmin_row(key + i * d, d, j1);
-    if (lane == 0) {
-      dm[i * d + j1] = 1;
-      dm[i * d + j2] = 1;
+  if (d <= 16) {
+    // one row per half-warp: a butterfly over the 16 lanes keeps the two
+    // smallest (key, j) pairs (ties -> smaller j)
+    const int h = lane >> 4, j = lane & 15;
+    for (int i0 = 2 * w; i0 < k; i0 += 2 * nw) {
+      const int i = i0 + h;
+      unsigned long long a1 = ~0ull, a2 = ~0ull;
+      int j1 = 0x7fff, j2 = 0x7fff;
+      if (i < k && j < d) {
+        a1 = key[i * d + j];
+        j1 = j;
+      }
+#pragma unroll
+      for (int o = 8; o > 0; o >>= 1) {
+        const unsigned long long b1 = __shfl_xor_sync(0xffffffffu, a1, o);
+        const unsigned long long b2 = __shfl_xor_sync(0xffffffffu, a2, o);
+        const int k1 = __shfl_xor_sync(0xffffffffu, j1, o);
+        const int k2 = __shfl_xor_sync(0xffffffffu, j2, o);
+        const bool bfirst = b1 < a1 || (b1 == a1 && k1 < j1);
+        // merged second = min(max(a1, b1), min(a2, b2))
+        unsigned long long hk = bfirst ? a1 : b1;
+        int hj = bfirst ? j1 : k1;
+        const bool b2first = b2 < a2 || (b2 == a2 && k2 < j2);
+        const unsigned long long lk2 = b2first ? b2 : a2;
+        const int lj2 = b2first ? k2 : j2;
+        if (lk2 < hk || (lk2 == hk && lj2 < hj)) {
+          hk = lk2;
+          hj = lj2;
+        }
+        if (bfirst) {
+          a1 = b1;
+          j1 = k1;
+        }
+        a2 = hk;
+        j2 = hj;
+      }
+      if (i < k && j == 0) {
+        dm[i * d + j1] = 1;
+        dm[i * d + j2] = 1;
+      }
+    }
+  } else {
+    for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
+      const int j1 = warp_argmin_row(key + i * d, d, -1);
+      const int j2 = warp_argmin_row(key + i * d, d, j1);
+      if (lane == 0) {
+        dm[i * d + j1] = 1;
+        dm[i * d + j2] = 1;
+      }
     }
   }
   __syncthreads();
   TST(T, 4);
   const int R = k * l - 2 * k;
-  if (R > 0 && kd <= 2048) {
+  if (R > 0 && kd <= 32 * nw) {
+    // every warp sorts 32 cells by (key, c) with a register bitonic network
+    // (taken / padding cells carry key ~0 and sort last), then each free cell's
+    // rank is its position in its own list plus a binary search in every other
+    // list: O(log) dependent steps instead of a scan over all k*d keys
+    unsigned long long* sk = (unsigned long long*)T.Z;  // [kd] sorted keys by list
+    int* si = (int*)T.dev;                              // [kd] their cells
+    const int nl = (kd + 31) >> 5;
+    unsigned long long kc = ~0ull;
+    int ic = 0x7fffffff;
+    if (w < nl) {
+      const int c = w * 32 + lane;
+      if (c < kd) {
+        kc = dm[c] ? ~0ull : key[c];
+        ic = c;
+      }
+#pragma unroll
+      for (int size = 2; size <= 32; size <<= 1) {
+#pragma unroll
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+          const unsigned long long ok = __shfl_xor_sync(0xffffffffu, kc, stride);
+          const int oi = __shfl_xor_sync(0xffffffffu, ic, stride);
+          const bool up = size == 32 || (lane & size) == 0;
+          const bool lower = (lane & stride) == 0;
+          const bool oless = ok < kc || (ok == kc && oi < ic);
+          if (lower == up ? oless : !oless) {
+            kc = ok;
+            ic = oi;
+          }
+        }
+      }
+    }
+    __syncthreads();  // every key is in a register: Z and the key array are free
+    if (w < nl && ic < kd) {  // padding (ic = INT_MAX) sorts last: lanes >= len
+      sk[w * 32 + lane] = kc;
+      si[w * 32 + lane] = ic;
+    }
+    __syncthreads();
+    if (w < nl && ic < kd && !dm[ic]) {
+      int rank = lane;
+#pragma unroll 4
+      for (int w2 = 0; w2 < nl; ++w2) {
+        if (w2 == w) continue;
+        const unsigned long long* lk = sk + w2 * 32;
+        const int* li = si + w2 * 32;
+        const int len = min(32, kd - w2 * 32);  // entries >= len: +inf
+        int b = 0;  // number of entries of list w2 before (kc, ic)
+#pragma unroll
+        for (int half = 16; half > 0; half >>= 1) {
+          const int t = b + half - 1;
+          if (t < len) {
+            const unsigned long long v = lk[t];
+            if (v < kc || (v == kc && li[t] < ic)) b += half;
+          }
+        }
+        if (b < len) {
+          const unsigned long long v = lk[b];
+          if (v < kc || (v == kc && li[b] < ic)) ++b;
+        }
+        rank += b;
+      }
+      if (rank < R) dm[ic] = 1;
+    }
+  } else if (R > 0 && kd <= 512) {  // rank by a scan over all keys: O(kd^2 / threads)
     for (int c = tid; c < kd; c += bd)
       if (dm[c]) key[c] = ~0ull;  // taken: never before a free cell
     __syncthreads();
@@ -1938,6 +2044,42 @@ __device__ __forceinline__ void band_sums_d16(const float* __restrict__ xs, int 
   }
 }
 
+// The same for d > 16: lane = dimension jb + lane of each 32-dimension block,
+// every lane walks the whole member mask of the slot (4-way bank conflicts
+// at the LD = P + 4 row stride instead of 32-way).
+__device__ __forceinline__ void band_sums_gen(const float* __restrict__ xs, int LD, int q0,
+                                              const float* __restrict__ med_s, int MS, int na,
+                                              int d, const unsigned* __restrict__ bal,
+                                              long long* __restrict__ acc,
+                                              const double* __restrict__ scale_s) {
+  const int lane = threadIdx.x & 31;
+  for (int jb = 0; jb < d; jb += 32) {
+    const int j = jb + lane;
+    const bool jv = j < d;
+    const float* xr = xs + (size_t)(jv ? j : 0) * LD + q0;
+    const double sc = scale_s[jv ? j : 0];
+    for (int a = 0; a < na; ++a) {
+      unsigned m = bal[a];
+      const double c = (double)med_s[a * MS + (jv ? j : 0)];
+      double s0 = 0.0, s1 = 0.0;
+      while (m) {
+        const int b0 = __ffs(m) - 1;
+        m &= m - 1u;
+        const float x0 = xr[b0];
+        if (m) {
+          const int b1 = __ffs(m) - 1;
+          m &= m - 1u;
+          const float x1 = xr[b1];
+          s1 = dadd(s1, fabs(dsub((double)x1, c)));
+        }
+        s0 = dadd(s0, fabs(dsub((double)x0, c)));
+      }
+      const double s = dadd(s0, s1);
+      if (jv && s != 0.0) acc[a * d + j] += __double2ll_rn(dmul(s, sc));
+    }
+  }
+}
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
 // One point per lane; the cached Dist rows of the active slots arrive through
 // the same TMA ring as the data (rows d..).  DR: coordinates in registers.
@@ -1958,7 +2100,6 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   ActSlot* act_s = SMP(ActSlot, act);
   int* row_s = SMP(int, row);
   double* scale_s = SMP(double, scale);
-  Cell* cells = SMP(Cell, cells);
   unsigned* bal_s = SMP(unsigned, bal);
   long long* acc_s = SMP(long long, acc);
   long long* cnt_s = SMP(long long, cnt);
@@ -1992,7 +2133,6 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
     const int a = e / MS, j = e - a * MS;
     const float m = j < d ? p.mrows[(long long)act_s[a].mpos * d + j] : 0.f;
     med_s[e] = m;
-    if (j < d) cells[a * d + j] = Cell{a, j, a * d + j, (double)m};
   }
   __syncthreads();
   long long nfb = 0;
@@ -2076,7 +2216,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
         if (DR == 16)
           band_sums_d16(xs, LD, w * 32, med_s, MS, na, d, bal, acc, scale_s);
         else
-          warp_cells<1, 1>(xs, LD, w * 32, cells, na * d, bal, acc, scale_s);
+          band_sums_gen(xs, LD, w * 32, med_s, MS, na, d, bal, acc, scale_s);
         pipe_release(R, stg);
       }
     }
@@ -3306,9 +3446,10 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     LB b;
     L.nw = nw1;
     L.P = P;
-    // d <= 16: rows padded by 4 floats so that the lane-per-dimension band
-    // sums of k_locality read a point's d coordinates from distinct banks
-    L.ldr = d <= 16 ? P + 4 : P;
+    // rows padded by 4 floats so that the lane-per-dimension band sums of
+    // k_locality read a point's coordinates with at most 2- (d <= 16) or
+    // 4-way bank conflicts
+    L.ldr = P + 4;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
     L.buf = b.take((size_t)stages * (d + k) * L.ldr * 4);
@@ -3316,7 +3457,6 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.act = b.take(sizeof(ActSlot) * KMAX);
     L.row = b.take(4 * KMAX);
     L.scale = b.take(8 * (size_t)d);
-    L.cells = b.take(sizeof(Cell) * kd);
     L.bal = b.take(4 * (size_t)nw1 * KMAX);
     L.acc = b.take(8 * (size_t)nw1 * kd);
     L.cnt = b.take(8 * (size_t)nw1 * KMAX);

@@ -67,6 +67,7 @@ SHAPES = [
     (4097, 33, 8, 6, 20, 5),
     (1500, 100, 10, 10, 20, 5),
     (3000, 64, 32, 3, 8, 2),
+    (2500, 100, 24, 5, 10, 3),  # k*d = 2400: radix selection of the tails
 ]
 
 
