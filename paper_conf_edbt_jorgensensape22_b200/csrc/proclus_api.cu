@@ -685,6 +685,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.tail_smem = ps.tail_smem;
   p.nchunks = (h->n + ps.P - 1) / ps.P;
   p.fuse_tail = h->world == 1 ? 1 : 0;
+  p.cost1 = ps.cost1;
   p.out_labels = h->out_labels.p;
   p.Delta = h->Delta.p;
   if (h->trace) {

@@ -80,8 +80,8 @@ struct TailLayout {
   int mrow, fall, uall, pall;  // rows of M and their tables, or mrow = -1
   int bytes;
 };
-enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3, KK_LS2 = 4, KK_REF2 = 5, KK_ASG2 = 6, KK_ASG3 = 7 };
-constexpr int NLAY = 8;
+enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3, KK_LS2 = 4, KK_REF2 = 5, KK_ASG2 = 6, KK_ASG3 = 7, KK_COST1 = 8 };
+constexpr int NLAY = 9;
 
 struct RunParams {
   long long n;        // rows on this device
@@ -115,6 +115,7 @@ struct RunParams {
   int stages;              // ring depth (2 or 3)
   long long nchunks;
   int fuse_tail;           // 1: last block finalises (single GPU)
+  int cost1;               // 1: the cost pass sums per cluster (k_cost1), cells 0..k-1
   int use_cond;            // 1: running inside a graph while-node
   unsigned long long cond; // cudaGraphConditionalHandle
   TraceBufs tr;

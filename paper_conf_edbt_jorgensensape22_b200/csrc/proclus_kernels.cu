@@ -1258,10 +1258,10 @@ __device__ __forceinline__ int warp_argmin_row(const unsigned long long* keys, i
 // selection of Alg 4 l.15-16 (reading R10): per medoid the two smallest by
 // (Z, j), then the k*l - 2k smallest of the rest by (Z, i, j).  The order is
 // taken on order-preserving 64-bit keys of Z (T.dev); the rest is selected by
-// sorted warp lists (k*d <= 32 * warps), a rank scan (k*d <= 512), else a
-// block-wide radix select (8 passes of 8-bit histograms).  Writes D as a mask (T.dm), |D_i|
+// rank scan (k*d <= 512), else a block-wide radix select (8 passes of
+// 8-bit histograms).  Writes D as a mask (T.dm), |D_i|
 // (S->nD) and, in global memory, the mask and the ascending dimension lists
-// used by the passes.  Needs X in T.X; clobbers T.Z and T.dev (keys / sorted lists).
+// used by the passes.  Needs X in T.X; clobbers T.Z and T.dev.
 __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   __shared__ double Ys[KMAX], Ss[KMAX];
   const int tid = threadIdx.x, bd = blockDim.x, lane = tid & 31, w = tid >> 5, nw = bd >> 5;
@@ -1304,124 +1304,18 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   }
   __syncthreads();
   TST(T, 3);
-  if (d <= 16) {
-    // one row per half-warp: a butterfly over the 16 lanes keeps the two
-    // smallest (key, j) pairs (ties -> smaller j)
-    const int h = lane >> 4, j = lane & 15;
-    for (int i0 = 2 * w; i0 < k; i0 += 2 * nw) {
-      const int i = i0 + h;
-      unsigned long long a1 = ~0ull, a2 = ~0ull;
-      int j1 = 0x7fff, j2 = 0x7fff;
-      if (i < k && j < d) {
-        a1 = key[i * d + j];
-        j1 = j;
-      }
-#pragma unroll
-      for (int o = 8; o > 0; o >>= 1) {
-        const unsigned long long b1 = __shfl_xor_sync(0xffffffffu, a1, o);
-        const unsigned long long b2 = __shfl_xor_sync(0xffffffffu, a2, o);
-        const int k1 = __shfl_xor_sync(0xffffffffu, j1, o);
-        const int k2 = __shfl_xor_sync(0xffffffffu, j2, o);
-        const bool bfirst = b1 < a1 || (b1 == a1 && k1 < j1);
-        // merged second = min(max(a1, b1), min(a2, b2))
-        unsigned long long hk = bfirst ? a1 : b1;
-        int hj = bfirst ? j1 : k1;
-        const bool b2first = b2 < a2 || (b2 == a2 && k2 < j2);
-        const unsigned long long lk2 = b2first ? b2 : a2;
-        const int lj2 = b2first ? k2 : j2;
-        if (lk2 < hk || (lk2 == hk && lj2 < hj)) {
-          hk = lk2;
-          hj = lj2;
-        }
-        if (bfirst) {
-          a1 = b1;
-          j1 = k1;
-        }
-        a2 = hk;
-        j2 = hj;
-      }
-      if (i < k && j == 0) {
-        dm[i * d + j1] = 1;
-        dm[i * d + j2] = 1;
-      }
-    }
-  } else {
-    for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
-      const int j1 = warp_argmin_row(key + i * d, d, -1);
-      const int j2 = warp_argmin_row(key + i * d, d, j1);
-      if (lane == 0) {
-        dm[i * d + j1] = 1;
-        dm[i * d + j2] = 1;
-      }
+  for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
+    const int j1 = warp_argmin_row(key + i * d, d, -1);
+    const int j2 = warp_argmin_row(key + i * d, d, j1);
+    if (lane == 0) {
+      dm[i * d + j1] = 1;
+      dm[i * d + j2] = 1;
     }
   }
   __syncthreads();
   TST(T, 4);
   const int R = k * l - 2 * k;
-  if (R > 0 && kd <= 32 * nw) {
-    // every warp sorts 32 cells by (key, c) with a register bitonic network
-    // (taken / padding cells carry key ~0 and sort last), then each free cell's
-    // rank is its position in its own list plus a binary search in every other
-    // list: O(log) dependent steps instead of a scan over all k*d keys
-    unsigned long long* sk = (unsigned long long*)T.Z;  // [kd] sorted keys by list
-    int* si = (int*)T.dev;                              // [kd] their cells
-    const int nl = (kd + 31) >> 5;
-    unsigned long long kc = ~0ull;
-    int ic = 0x7fffffff;
-    if (w < nl) {
-      const int c = w * 32 + lane;
-      if (c < kd) {
-        kc = dm[c] ? ~0ull : key[c];
-        ic = c;
-      }
-#pragma unroll
-      for (int size = 2; size <= 32; size <<= 1) {
-#pragma unroll
-        for (int stride = size >> 1; stride > 0; stride >>= 1) {
-          const unsigned long long ok = __shfl_xor_sync(0xffffffffu, kc, stride);
-          const int oi = __shfl_xor_sync(0xffffffffu, ic, stride);
-          const bool up = size == 32 || (lane & size) == 0;
-          const bool lower = (lane & stride) == 0;
-          const bool oless = ok < kc || (ok == kc && oi < ic);
-          if (lower == up ? oless : !oless) {
-            kc = ok;
-            ic = oi;
-          }
-        }
-      }
-    }
-    __syncthreads();  // every key is in a register: Z and the key array are free
-    if (w < nl && ic < kd) {  // padding (ic = INT_MAX) sorts last: lanes >= len
-      sk[w * 32 + lane] = kc;
-      si[w * 32 + lane] = ic;
-    }
-    __syncthreads();
-    if (w < nl && ic < kd && !dm[ic]) {
-      int rank = lane;
-#pragma unroll 4
-      for (int w2 = 0; w2 < nl; ++w2) {
-        if (w2 == w) continue;
-        const unsigned long long* lk = sk + w2 * 32;
-        const int* li = si + w2 * 32;
-        const int len = min(32, kd - w2 * 32);  // entries >= len: +inf
-        int b = 0;  // number of entries of list w2 before (kc, ic)
-#pragma unroll
-        for (int half = 16; half > 0; half >>= 1) {
-          const int t = b + half - 1;
-          if (t < len) {
-            const unsigned long long v = lk[t];
-            if (v < kc || (v == kc && li[t] < ic)) b += half;
-          }
-        }
-        if (b < len) {
-          const unsigned long long v = lk[b];
-          if (v < kc || (v == kc && li[b] < ic)) ++b;
-        }
-        rank += b;
-      }
-      if (rank < R) dm[ic] = 1;
-    }
-  } else if (R > 0 && kd <= 512) {  // rank by a scan over all keys: O(kd^2 / threads)
+  if (R > 0 && kd <= 512) {  // rank by a scan over all keys: O(kd^2 / threads)
     for (int c = tid; c < kd; c += bd)
       if (dm[c]) key[c] = ~0ull;  // taken: never before a free cell
     __syncthreads();
@@ -1736,6 +1630,7 @@ __device__ void tail_assign(const RunParams& p, TailMem& T) {
 // trip brings the state, the deviation sums, the dimension lists, 2^-e_j and
 // (when cached) the rows of M with their DistFound / delta' entries, so the
 // prologue of the next iteration needs no further global loads.
+__device__ int cost_qexp(const double* sc, int sgn, const int* dl, const int* nD, int k, int d);
 __device__ void tail_cost(const RunParams& p, TailMem& T) {
   DevState* S = T.S;
   const int k = p.k, d = p.d, kd = k * d, nM = p.nM;
@@ -1746,7 +1641,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
   state_issue(p, sr);
   for (int c = tid; c < kd; c += bd) {
     const int dl = p.dlist[c];
-    const long long v = take_acc(p, c);
+    const long long v = (!p.cost1 || c < k) ? take_acc(p, c) : 0ll;
     T.dl[c] = dl;
     raw[c] = v;
   }
@@ -1762,27 +1657,36 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
   state_commit(p, sr, S);
   __syncthreads();
   TST(T, 10);
-  for (int c = tid; c < kd; c += bd) {  // dev_it and the per-term quotients of eq 1
-    const int i = c / d, t = c - i * d;
-    const long long ci = S->sizes[i];
-    const bool on = t < S->nD[i];
-    const double dv = on ? dmul((double)raw[c], T.isc[T.dl[c]]) : 0.0;
-    T.dev[c] = dv;
-    T.Z[c] = (on && ci != 0) ? ddiv(dv, (double)ci) : 0.0;
-  }
-  __syncthreads();
-  if (tid < k) {  // |C_i| * w_i of eq 1, terms added in t order
-    const int i = tid;
-    const long long c = S->sizes[i];
-    double cw = 0.0;
-    if (c != 0) {
-      double wv = 0.0;
-      const int nd = S->nD[i];
-      for (int t = 0; t < nd; ++t) wv = dadd(wv, T.Z[i * d + t]);
-      wv = ddiv(wv, (double)nd);
-      cw = dmul((double)c, wv);
+  if (p.cost1) {  // |C_i| w_i = (sum_t dev_it) / |D_i| (eq 1 with eq 2's weight)
+    const int ec = cost_qexp(T.isc, -1, T.dl, S->nD, k, d);
+    if (tid < k) {
+      const int i = tid;
+      const long long c = S->sizes[i];
+      cw_s[i] = c != 0 ? ddiv(scalbn((double)raw[i], -ec), (double)S->nD[i]) : 0.0;
     }
-    cw_s[i] = cw;
+  } else {
+    for (int c = tid; c < kd; c += bd) {  // dev_it and the per-term quotients of eq 1
+      const int i = c / d, t = c - i * d;
+      const long long ci = S->sizes[i];
+      const bool on = t < S->nD[i];
+      const double dv = on ? dmul((double)raw[c], T.isc[T.dl[c]]) : 0.0;
+      T.dev[c] = dv;
+      T.Z[c] = (on && ci != 0) ? ddiv(dv, (double)ci) : 0.0;
+    }
+    __syncthreads();
+    if (tid < k) {  // |C_i| * w_i of eq 1, terms added in t order
+      const int i = tid;
+      const long long c = S->sizes[i];
+      double cw = 0.0;
+      if (c != 0) {
+        double wv = 0.0;
+        const int nd = S->nD[i];
+        for (int t = 0; t < nd; ++t) wv = dadd(wv, T.Z[i * d + t]);
+        wv = ddiv(wv, (double)nd);
+        cw = dmul((double)c, wv);
+      }
+      cw_s[i] = cw;
+    }
   }
   __syncthreads();
   TST(T, 11);
@@ -2896,6 +2800,119 @@ __global__ void __launch_bounds__(416) k_lsum2(RunParams p) {
   }
 }
 
+
+// --- EvaluateCluster (Alg 6, eq 9) with per-cluster sums.  The cost only
+// needs, per cluster i, sum_{t < |D_i|} sum_{p in C_i} |x_pj - mu_ij| (the
+// division by |C_i| of eq 1 cancels against the weight |C_i| of eq 2), so
+// every term is quantised on its own at ONE scale 2^e_c (cost_qexp) and a
+// point's |D_c| terms go into a lane-private int64 accumulator of its
+// cluster (a shared-memory column per lane): no sort, no ballot, no barrier
+// in the chunk loop, one table entry + one ring read + 4 DP ops per term.
+// The integer totals do not depend on the order, the grid or the GPU count.
+struct __align__(16) CItem {
+  int joff;   // byte offset of dimension row j in a ring stage
+  int pad;
+  double cq;  // mu_ij * 2^e_c (exact: power-of-two scale)
+};
+
+// e_c = min e_j over the dimensions of D minus hb, 2^hb >= max |D_i|: one
+// dimension's total stays < 2^(61 - hb) (proclus_api.cu), a cluster's sum
+// over its <= 2^hb dimensions < 2^61, and one term < 2^51 (q_abs).  Block-
+// wide (one cell per thread, shared-memory min / max); sc[j] = 2^(sgn e_j).
+__device__ int cost_qexp(const double* sc, int sgn, const int* dl, const int* nD, int k, int d) {
+  __shared__ int emin_s, ndmax_s;
+  if (threadIdx.x == 0) {
+    emin_s = 1 << 20;
+    ndmax_s = 1;
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD[i]) atomicMin(&emin_s, sgn * ilogb(sc[dl[e]]));
+    if (t == 0) atomicMax(&ndmax_s, nD[i]);
+  }
+  __syncthreads();
+  const int r = emin_s - (32 - __clz(ndmax_s));
+  __syncthreads();
+  return r;
+}
+
+__global__ void __launch_bounds__(288) k_cost1(RunParams p) {
+  DevState* st = p.st;
+  if (st->done) return;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_COST1];
+#define LAYK KK_COST1
+  const int P = p.P, d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const Pipe R = pipe_of(L, smraw, d);
+  CItem* tab = SMP(CItem, tab);
+  int* nD_s = SMP(int, nD);
+  long long* acc_s = SMP(long long, acc);  // [nw][k][32] lane-private columns
+  const unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  const long long nmy = chunks_of_block(p);
+  for (int i = threadIdx.x; i < k; i += blockDim.x) nD_s[i] = st->nD[i];
+  for (int e = threadIdx.x; e < nw * k * 32; e += blockDim.x) acc_s[e] = 0;
+  pipe_init(p, R, nw);
+  __syncthreads();
+  const double sc = scalbn(1.0, cost_qexp(p.scale, 1, p.dlist, nD_s, k, d));
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i]) tab[e] = CItem{p.dlist[e] * R.ldr * 4, 0, dmul(p.mu[e], sc)};
+  }
+  __syncthreads();
+  if (w == nw) {
+    pipe_produce(p, R, nmy, lab, nullptr);
+  } else {
+    long long* acc = acc_s + (size_t)w * k * 32 + lane;
+    const int q = w * 32 + lane;
+    long long gp = (long long)blockIdx.x * P + q;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      mbar_wait(&R.full[stg], rp.ph);
+      if (gp < p.n) {
+        const int c = R.lab[(size_t)stg * P + q];
+        const char* xq = reinterpret_cast<const char*>(R.buf + (size_t)stg * R.rows * R.ldr + q);
+        const CItem* tb = tab + c * d;
+        const int nd = nD_s[c];
+        long long a0 = 0, a1 = 0;
+        int t = 0;
+        for (; t + 2 <= nd; t += 2) {
+          const CItem e0 = tb[t], e1 = tb[t + 1];
+          const float x0 = *reinterpret_cast<const float*>(xq + e0.joff);
+          const float x1 = *reinterpret_cast<const float*>(xq + e1.joff);
+          a0 += q_abs(x0, sc, e0.cq);
+          a1 += q_abs(x1, sc, e1.cq);
+        }
+        if (t < nd) {
+          const CItem e0 = tb[t];
+          a0 += q_abs(*reinterpret_cast<const float*>(xq + e0.joff), sc, e0.cq);
+        }
+        acc[c * 32] += a0 + a1;
+      }
+      pipe_release(R, stg);
+    }
+  }
+  __syncthreads();
+  {  // per cluster: warps, then lanes; one atomic per block and cluster
+    const int cp = blockIdx.x % NCOPY;
+    for (int c = w; c < k; c += nw + 1) {
+      long long s = 0;
+      for (int ww = 0; ww < nw; ++ww) s += acc_s[((size_t)ww * k + c) * 32 + lane];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+      if (lane == 0 && s)
+        atomicAdd((unsigned long long*)&p.accg[(size_t)cp * k * d + c], (unsigned long long)s);
+    }
+  }
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[2])) return;
+  RUN_TAIL(tail_cost, 2);
+#undef LAYK
+}
+
 // --- AssignPoints (Alg 5) + centroid sums (Alg 6 l.1-8), d <= 16: every
 // lane holds the 16 coordinates of 2 point PAIRS in registers (LDS.64 once
 // per pair and dimension) and evaluates seg_{D_c} for all clusters with
@@ -3615,6 +3632,25 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     ps.tpb_asg2 = 32 * (nw + 1);
     ps.smem_asg2 = ps.asg2 ? ps.lay[KK_ASG2].bytes : 0;
   }
+  {  // per-cluster cost pass (k_cost1): lane-private columns [nw][k][32]
+    SmemLayout L = blank_layout();
+    LB b;
+    L.nw = nw1;
+    L.P = P;
+    L.ldr = P;  // a lane reads its own point: conflict-free whatever the row
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * d * P * 4);
+    L.lab = b.take((size_t)stages * P);
+    L.tab = b.take(sizeof(CItem) * kd);
+    L.nD = b.take(4 * KMAX);
+    L.acc = b.take(8 * (size_t)nw1 * k * 32);
+    finish(L, b, ps.tl);
+    ps.lay[KK_COST1] = L;
+    ps.cost1 = L.bytes <= 200 * 1024 && !getenv("PROCLUS_OLD_COST");
+    ps.tpb_cost1 = 32 * (nw1 + 1);
+    ps.smem_cost1 = ps.cost1 ? L.bytes : 0;
+  }
   ps.smem_loc = ps.lay[KK_LOC].bytes;
   ps.smem_asg = ps.lay[KK_ASG].bytes;
   ps.smem_cost = ps.lay[KK_LSUM].bytes;
@@ -3655,6 +3691,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   ps.grid_ref2 = ps.ref2 ? grid_of((const void*)k_lsum2<1>, ps.smem_ref2, ps.tpb_ref2) : 0;
   ps.grid_asg2 = ps.asg2 ? grid_of((const void*)k_assign2, ps.smem_asg2, ps.tpb_asg2) : 0;
   ps.grid_asg3 = ps.asg3 ? grid_of((const void*)k_assign3, ps.smem_asg3, ps.tpb_asg3) : 0;
+  ps.grid_cost1 = ps.cost1 ? grid_of((const void*)k_cost1, ps.smem_cost1, ps.tpb_cost1) : 0;
   ps.grid = ps.grid_loc;
   ps.per_sm = ps.grid_loc / num_sms;
   return ps;
@@ -3688,6 +3725,11 @@ cudaError_t configure_kernels(const PassShape& ps) {
                              (int)ps.smem_asg2);
     if (e != cudaSuccess) return e;
   }
+  if (ps.cost1) {
+    e = cudaFuncSetAttribute((const void*)k_cost1, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)ps.smem_cost1);
+    if (e != cudaSuccess) return e;
+  }
   if (ps.asg3) {
     e = cudaFuncSetAttribute((const void*)k_assign3, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)ps.smem_asg3);
@@ -3713,7 +3755,9 @@ void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  if (ps.lsum2)
+  if (ps.cost1)
+    k_cost1<<<ps.grid_cost1, ps.tpb_cost1, ps.smem_cost1, s>>>(p);
+  else if (ps.lsum2)
     k_lsum2<0><<<ps.grid_ls2, ps.tpb_ls2, ps.smem_ls2, s>>>(p);
   else
     k_labelsum<0><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_cost, s>>>(p);
