@@ -1146,7 +1146,17 @@ __shared__ unsigned long long g_tst_last;
       g_tst_last = t_;                                     \
     }                                                      \
   } while (0)
+#define TSTW_DECL() unsigned long long tw_last_ = clock64()
+#define TSTW(T, idx)                                                  \
+  do {                                                                \
+    __syncwarp();                                                     \
+    const unsigned long long t_ = clock64();                          \
+    if ((threadIdx.x & 31) == 0) (T).S->dbg_cyc[idx] += t_ - tw_last_; \
+    tw_last_ = t_;                                                    \
+  } while (0)
 #else
+#define TSTW_DECL() do {} while (0)
+#define TSTW(T, idx) do {} while (0)
 #define TST_START() \
   do {              \
   } while (0)
@@ -1262,7 +1272,7 @@ __device__ __forceinline__ int warp_argmin_row(const unsigned long long* keys, i
 // 8-bit histograms).  Writes D as a mask (T.dm), |D_i|
 // (S->nD) and, in global memory, the mask and the ascending dimension lists
 // used by the passes.  Needs X in T.X; clobbers T.Z and T.dev.
-__device__ void zscore_select_s(const RunParams& p, TailMem& T) {
+__device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
   __shared__ double Ys[KMAX], Ss[KMAX];
   const int tid = threadIdx.x, bd = blockDim.x, lane = tid & 31, w = tid >> 5, nw = bd >> 5;
   const int k = p.k, d = p.d, l = p.l, kd = k * d;
@@ -1293,7 +1303,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     Ss[tid] = __dsqrt_rn(ddiv(s2, (double)(d - 1)));
   }
   __syncthreads();
-  TST(T, 2);
+  TST(T, tq < 0 ? 2 : tq);
   for (int c = tid; c < kd; c += bd) {
     const int i = c / d;
     const double sg = Ss[i];
@@ -1303,7 +1313,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     dm[c] = 0;
   }
   __syncthreads();
-  TST(T, 3);
+  TST(T, tq < 0 ? 3 : tq);
   for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
     const int j1 = warp_argmin_row(key + i * d, d, -1);
     const int j2 = warp_argmin_row(key + i * d, d, j1);
@@ -1313,7 +1323,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     }
   }
   __syncthreads();
-  TST(T, 4);
+  TST(T, tq < 0 ? 4 : tq);
   const int R = k * l - 2 * k;
   if (R > 0 && kd <= 512) {  // rank by a scan over all keys: O(kd^2 / threads)
     for (int c = tid; c < kd; c += bd)
@@ -1418,7 +1428,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
     }
   }
   __syncthreads();
-  TST(T, 6);
+  TST(T, tq < 0 ? 6 : tq);
   for (int i = w; i < k; i += nw) {  // |D_i| and the ascending lists, one warp per row
     int base = 0;
     for (int j0 = 0; j0 < d; j0 += 32) {
@@ -1432,7 +1442,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T) {
   }
   for (int c = tid; c < kd; c += bd) p.dmask[c] = dm[c];
   __syncthreads();
-  TST(T, 7);
+  TST(T, tq < 0 ? 7 : tq);
 }
 
 // ------------------------------------------------------------ iteration prologue
@@ -1691,6 +1701,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
   __syncthreads();
   TST(T, 11);
   if (tid < 32) {  // control, one warp
+    TSTW_DECL();
     const unsigned full = 0xffffffffu;
     double cost = 0.0;
     if (lane == 0) {
@@ -1718,6 +1729,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
       }
     }
     __syncwarp();
+    TSTW(T, 12);
     // bad medoids (R11): |C_i| < n/k * minDev in CBest, else the smallest
     const double thr = dmul(ddiv((double)p.n_total, (double)k), p.minDev);
     const long long sb = lane < k ? S->sizes_best[lane] : 0ll;
@@ -1740,6 +1752,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
     }
     if (lane < k) S->mcur[lane] = S->mbest[lane];
     __syncwarp();
+    TSTW(T, 13);
     // pool = ascending positions of M not in MBest
     int np = 0;
     for (int t0 = 0; t0 < nM; t0 += 32) {
@@ -1752,6 +1765,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
       np += __popc(b);
     }
     __syncwarp();
+    TSTW(T, 18);
     // replacement draws (stream IT): the r-th remaining pool entry, in order;
     // every lane runs the same generator, the removal shift is warp-wide
     unsigned long long rng = S->rng;
@@ -1768,12 +1782,14 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
       }
       --np;
     }
+    TSTW(T, 19);
     if (lane == 0) {
       S->rng = rng;
       S->done = (S->itr >= p.itrPat || S->iterations >= p.max_iter) ? 1 : 0;
       if (p.use_cond)
         cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, S->done ? 0u : 1u);
     }
+    TSTW(T, 22);
   }
   __syncthreads();
   TST(T, 14);
@@ -2040,6 +2056,8 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   }
   __syncthreads();
   long long nfb = 0;
+  int ncomp = 0;  // active slots whose Dist row is computed in this pass
+  for (int a = 0; a < na; ++a) ncomp += row_s[a] < 0;
   if (na > 0) {
     if (w == nw) {
       pipe_produce(p, R, nmy, nullptr, ex);
@@ -2057,7 +2075,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
         const float* xs = R.buf + (size_t)stg * R.rows * LD;
         const bool valid = gp < p.n;
         float xr[DR > 0 ? DR : 1];
-        if (DR > 0) {
+        if (DR > 0 && ncomp > 0) {  // coordinates only when a Dist row is computed
 #pragma unroll
           for (int j = 0; j < DR; ++j) xr[j] = (j < d) ? xs[j * LD + q] : 0.f;
         }

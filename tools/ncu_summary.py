@@ -87,15 +87,21 @@ for r in data:
         rec[k] = round(val, 3)
     full.append(rec)
 
-traffic = {}
+traffic, tcount = {}, {}
 for rec in full:
-    base = re.sub(r"<.*", "", rec["kernel"]).replace("k_", "")
-    name = {"labelsum": "cost", "greedy": "greedy", "sdist": "greedy"}.get(base, base)
-    if "dram_rd_MB" in rec and name not in traffic:
-        traffic[name] = (rec["dram_rd_MB"] + rec.get("dram_wr_MB", 0.0)) * 1e6
+    kname = rec["kernel"]
+    base = re.sub(r"<.*", "", kname).replace("k_", "")
+    if base in ("lsum2", "labelsum"):
+        base = "refine_x" if "<1>" in kname else "cost"
+    name = {"cost1": "cost", "greedy_cluster": "greedy", "sdist": "greedy"}.get(base, base)
+    if "dram_rd_MB" in rec:
+        traffic[name] = traffic.get(name, 0.0) + (rec["dram_rd_MB"] + rec.get("dram_wr_MB", 0.0)) * 1e6
+        tcount[name] = tcount.get(name, 0) + 1
+traffic = {kk: v / tcount[kk] for kk, v in traffic.items()}
 with open(os.path.join(prof, "ncu_traffic.json"), "w") as f:
-    json.dump({"source": f"profiles/{tag}_ncu_summary.md (ncu --set full, cold L2, first "
-                         f"launch of each kernel)", **traffic}, f, indent=1)
+    json.dump({"source": f"profiles/{tag}_ncu_summary.md (ncu --set full, cold L2, mean "
+                         f"dram read+write bytes per launch over the captured launches)",
+               **traffic}, f, indent=1)
 
 with open(os.path.join(prof, f"{tag}_ncu_summary.md"), "w") as f:
     f.write(f"# ncu summary, {tag}\n\n")

@@ -15,6 +15,6 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv \
     --log-file $OUT/launches.csv python bench.py --steps 2 --warmup 3 \
     --no-cpu-baseline --no-e2e > $OUT/launches_bench.log 2>&1
 ncu --set full --clock-control none --import-source on \
-    -k regex:"k_(locality|assign|labelsum|final|greedy|sdist)" -s 0 -c 12 \
+    -k regex:"k_(locality|assign|cost1|lsum2|labelsum|final|greedy|sdist)" -s 0 -c 16 \
     -o $OUT/full python tools/profile_run.py C3 1 > $OUT/full.log 2>&1
 ls -la $OUT
