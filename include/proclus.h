@@ -150,6 +150,17 @@ PROCLUS_API proclus_status proclus_create_ex(const float* data, int64_t n, int32
  * device pointer per the handle's options).  Drops all cached distances. */
 PROCLUS_API proclus_status proclus_load(proclus_handle* h, const float* data);
 
+/* Start copying the NEXT dataset `data` (host pointer, row-major n x d fp32
+ * of the handle's shape; pinned memory makes the copy asynchronous) into the
+ * handle's staging buffer on a separate copy stream and return at once, so
+ * that the transfer overlaps the clustering a following proclus_run performs
+ * on the current data.  A later proclus_load(h, data) with the same pointer
+ * waits for that copy instead of copying again.  The caller keeps `data`
+ * alive and unmodified until that proclus_load returns.  Nothing of the
+ * current data or its results changes.
+ * EINVAL: NULL arguments, a handle created with device-resident data. */
+PROCLUS_API proclus_status proclus_prefetch(proclus_handle* h, const float* data);
+
 /* One PROCLUS clustering (Alg 1): initialization (sample of A*k points,
  * Greedy to B*k potential medoids), iterative phase (Alg 1
  * l.5-14, with the FAST caches of section 3), refinement (Alg 1

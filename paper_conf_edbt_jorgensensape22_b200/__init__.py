@@ -72,6 +72,7 @@ SIGNATURES = [
     ("proclus_create_ex", C.c_int, [C.c_void_p, C.c_int64, C.c_int32,
                                     C.POINTER(proclus_options), C.POINTER(C.c_void_p)]),
     ("proclus_load", C.c_int, [C.c_void_p, C.c_void_p]),
+    ("proclus_prefetch", C.c_int, [C.c_void_p, C.c_void_p]),
     ("proclus_run", C.c_int, [C.c_void_p, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
                               C.c_double, C.c_int32, C.c_uint64, C.POINTER(proclus_result)]),
     ("proclus_run_multi", C.c_int, [C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p, C.c_int32,
@@ -137,6 +138,10 @@ def proclus_create(data, n: int, d: int) -> C.c_void_p:
 
 def proclus_load(h, data):
     _check(lib().proclus_load(h, C.c_void_p(_ptr(data))))
+
+
+def proclus_prefetch(h, data):
+    _check(lib().proclus_prefetch(h, C.c_void_p(_ptr(data))))
 
 
 def proclus_run(h, k, l, A, B, minDev, itrPat, seed, res: proclus_result):
@@ -262,6 +267,11 @@ class Proclus:
         if not hasattr(data, "data_ptr"):
             data = np.ascontiguousarray(data, dtype=np.float32)
         proclus_load(self.h, data)
+
+    def prefetch(self, data):
+        """Start the H2D copy of the next dataset (keep `data` alive and
+        unchanged until load(data) returns); load(data) then waits for it."""
+        proclus_prefetch(self.h, data)
 
     def _result_struct(self, k, labels=None):
         on_dev = labels is not None and hasattr(labels, "is_cuda") and bool(labels.is_cuda)

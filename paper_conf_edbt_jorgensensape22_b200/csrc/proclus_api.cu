@@ -116,6 +116,10 @@ struct proclus_handle {
   int64_t launches = 0;
 
   DBuf<float> xs, staging;
+  // proclus_prefetch: H2D of the next dataset into `staging` on cstream
+  cudaStream_t cstream = nullptr;
+  cudaEvent_t pf_done = nullptr, pack_done = nullptr;
+  const float* pf_src = nullptr;
   DBuf<int> flag;
   DBuf<unsigned> colmax;
   DBuf<double> scale, iscale;
@@ -229,7 +233,10 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
   const float* src = data;
   if (!h->data_on_device) {
     CK(h->staging.ensure((size_t)h->n * h->d));
-    CK(cudaMemcpyAsync(h->staging.p, data, bytes, cudaMemcpyHostToDevice, h->stream));
+    if (h->pf_src) CK(cudaStreamWaitEvent(h->stream, h->pf_done, 0));  // staging is being filled
+    if (h->pf_src != data)
+      CK(cudaMemcpyAsync(h->staging.p, data, bytes, cudaMemcpyHostToDevice, h->stream));
+    h->pf_src = nullptr;
     src = h->staging.p;
   }
   CK(cudaMemsetAsync(h->flag.p, 0, sizeof(int), h->stream));
@@ -238,6 +245,7 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
     launch_pack_soa(src, h->n, h->d, h->n_pad, h->xs.p, h->flag.p, h->colmax.p, h->stream);
   });
   CK(cudaGetLastError());
+  if (h->pack_done) CK(cudaEventRecord(h->pack_done, h->stream));  // staging read
   TRY(allreduce(h, h->colmax.p, h->d, ncclUint32, ncclMax));
   TRY(allreduce(h, h->flag.p, 1, ncclInt32, ncclMax));
   int bad = 0;
@@ -363,10 +371,36 @@ proclus_status proclus_load(proclus_handle* h, const float* data) {
   return upload_data(h, data);
 }
 
+proclus_status proclus_prefetch(proclus_handle* h, const float* data) {
+  if (!h || !data) return fail(PROCLUS_EINVAL, "NULL argument");
+  if (h->data_on_device) return fail(PROCLUS_EINVAL, "prefetch needs host-resident data");
+  TRY(set_device(h));
+  if (!h->cstream) {
+    CK(cudaStreamCreateWithFlags(&h->cstream, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&h->pf_done, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&h->pack_done, cudaEventDisableTiming));
+    CK(cudaEventRecord(h->pack_done, h->stream));
+  }
+  CK(h->staging.ensure((size_t)h->n * h->d));
+  if (h->pf_src) CK(cudaStreamWaitEvent(h->cstream, h->pf_done, 0));
+  CK(cudaStreamWaitEvent(h->cstream, h->pack_done, 0));  // the last pack has read staging
+  CK(cudaMemcpyAsync(h->staging.p, data, sizeof(float) * (size_t)h->n * h->d,
+                     cudaMemcpyHostToDevice, h->cstream));
+  CK(cudaEventRecord(h->pf_done, h->cstream));
+  h->pf_src = data;
+  return PROCLUS_OK;
+}
+
 void proclus_destroy(proclus_handle* h) {
   if (!h) return;
   cudaSetDevice(h->dev);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->cstream) {
+    cudaStreamSynchronize(h->cstream);
+    cudaStreamDestroy(h->cstream);
+    cudaEventDestroy(h->pf_done);
+    cudaEventDestroy(h->pack_done);
+  }
   if (h->gexec) cudaGraphExecDestroy(h->gexec);
   h->xs.release();
   h->staging.release();
@@ -478,8 +512,8 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   CK(h->gscratch.ensure(greedy_scratch_doubles((int)nS)));
   CK(h->mrows.ensure((size_t)nM * d));
   CK(h->mids.ensure((size_t)nM));
-  CK(cudaMemcpyAsync(h->sids.p, S.data(), sizeof(long long) * nS, cudaMemcpyHostToDevice,
-                     h->stream));
+  launch_put(h->sids.p, S.data(), sizeof(long long) * nS, h->stream);
+  CK(cudaGetLastError());
   launch(h, K_GATHER, -1, [&] {
     launch_gather_rows(h->xs.p, h->n_pad, d, h->sids.p, h->row_offset, h->n, (int)nS,
                        h->srows.p, h->stream);
@@ -639,7 +673,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   s.cost_best = INFINITY;
   s.cur_buf = 0;
   s.best_buf = 1;
-  CK(cudaMemcpyAsync(h->st.p, &s, sizeof(DevState), cudaMemcpyHostToDevice, h->stream));
+  launch_put(h->st.p, &s, sizeof(DevState), h->stream);
+  CK(cudaGetLastError());
   CK(cudaMemsetAsync(h->accg.p, 0, sizeof(long long) * NCOPY * KMAX * d, h->stream));
   CK(cudaMemsetAsync(h->cntg.p, 0, sizeof(long long) * NCOPY * KMAX, h->stream));
 

@@ -74,42 +74,75 @@ __device__ __forceinline__ void fence_mbar_init() {
 // ===================================================================== N0
 // row-major [n][d] -> SoA [d][n_pad] (zero padding), non-finite flag and the
 // per-dimension max |x| (as float bits; non-negative floats order as uints).
+// 32 x 32 tiles through shared memory; a block transposes PACK_TILES tiles of
+// consecutive points so that max |x_j| is reduced in the block first (one
+// atomicMax per column per block: the per-thread atomics on d addresses
+// serialised the whole pack).
+constexpr int PACK_TILES = 8;
 __global__ void k_pack_soa(const float* __restrict__ in, long long n, int d,
                            long long n_pad, float* __restrict__ xs, int* bad,
                            unsigned* colmax) {
   __shared__ float tile[32][33];
-  const long long p0 = (long long)blockIdx.x * 32;
+  __shared__ float red[8][33];
   const int j0 = blockIdx.y * 32;
   const int tx = threadIdx.x, ty = threadIdx.y;
   int nonfinite = 0;
   float amax = 0.f;
-  for (int r = ty; r < 32; r += 8) {
-    long long p = p0 + r;
-    int j = j0 + tx;
-    float v = 0.f;
-    if (p < n && j < d) {
-      v = in[p * d + j];
-      if (!isfinite(v))
-        nonfinite = 1;
-      else
-        amax = fmaxf(amax, fabsf(v));
+  for (int tt = 0; tt < PACK_TILES; ++tt) {
+    const long long p0 = ((long long)blockIdx.x * PACK_TILES + tt) * 32;
+    if (p0 >= n_pad) break;
+    for (int r = ty; r < 32; r += 8) {
+      const long long p = p0 + r;
+      const int j = j0 + tx;
+      float v = 0.f;
+      if (p < n && j < d) {
+        v = in[p * d + j];
+        if (!isfinite(v))
+          nonfinite = 1;
+        else
+          amax = fmaxf(amax, fabsf(v));
+      }
+      tile[r][tx] = v;
     }
-    tile[r][tx] = v;
+    __syncthreads();
+    for (int r = ty; r < 32; r += 8) {
+      const int j = j0 + r;
+      const long long p = p0 + tx;
+      if (j < d && p < n_pad) xs[(long long)j * n_pad + p] = tile[tx][r];
+    }
+    __syncthreads();
   }
   if (nonfinite) atomicOr(bad, 1);
-  if (j0 + tx < d && amax > 0.f) atomicMax(colmax + j0 + tx, __float_as_uint(amax));
+  red[ty][tx] = amax;
   __syncthreads();
-  for (int r = ty; r < 32; r += 8) {
-    int j = j0 + r;
-    long long p = p0 + tx;
-    if (j < d && p < n_pad) xs[(long long)j * n_pad + p] = tile[tx][r];
+  if (ty == 0) {
+    float m = red[0][tx];
+    for (int r = 1; r < 8; ++r) m = fmaxf(m, red[r][tx]);
+    if (j0 + tx < d && m > 0.f) atomicMax(colmax + j0 + tx, __float_as_uint(m));
   }
 }
 
 void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
                      unsigned* colmax, cudaStream_t s) {
-  dim3 grid((unsigned)((n_pad + 31) / 32), (unsigned)((d + 31) / 32));
+  dim3 grid((unsigned)((n_pad + 32 * PACK_TILES - 1) / (32 * PACK_TILES)), (unsigned)((d + 31) / 32));
   k_pack_soa<<<grid, dim3(32, 8), 0, s>>>(in, n, d, n_pad, xs, bad, colmax);
+}
+
+// Small host -> device uploads as kernel parameters (no copy-engine work, so
+// they never queue behind a proclus_prefetch transfer of the next dataset).
+struct Blob {
+  unsigned char b[BLOB_BYTES];
+};
+__global__ void k_put(unsigned char* __restrict__ dst, Blob src, int bytes) {
+  for (int i = threadIdx.x; i < bytes; i += blockDim.x) dst[i] = src.b[i];
+}
+void launch_put(void* dst, const void* src, size_t bytes, cudaStream_t s) {
+  for (size_t off = 0; off < bytes; off += BLOB_BYTES) {
+    Blob b;
+    const size_t n = bytes - off < (size_t)BLOB_BYTES ? bytes - off : (size_t)BLOB_BYTES;
+    memcpy(b.b, (const unsigned char*)src + off, n);
+    k_put<<<1, 256, 0, s>>>((unsigned char*)dst + off, b, (int)n);
+  }
 }
 
 __global__ void k_gather_rows(const float* __restrict__ xs, long long n_pad, int d,

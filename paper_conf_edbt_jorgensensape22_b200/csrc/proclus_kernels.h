@@ -50,6 +50,10 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
 void launch_gather_m(const float* srows, const long long* sids, const int* spos, int nM, int d,
                      float* mrows, long long* mids, cudaStream_t s);
 
+// Small H2D upload through kernel parameters (chunks of BLOB_BYTES).
+constexpr int BLOB_BYTES = 3968;
+void launch_put(void* dst, const void* src, size_t bytes, cudaStream_t s);
+
 PassShape pass_shape(int d, int k, int l, int nM, int num_sms);
 cudaError_t configure_kernels(const PassShape& ps);
 

@@ -158,6 +158,28 @@ def test_load_replaces_data(pk, orc):
     assert_parity(g, orc.proclus(d2, 5, 3, seed=1), what="after load")
 
 
+def test_prefetch_overlaps_next_dataset(pk, orc):
+    """proclus_prefetch stages the next dataset while the current one is
+    clustered; load() of the same pointer then swaps it in (P:87 per step)."""
+    import torch
+
+    a = synth.generate(3000, 9, 4, 3, seed=31)
+    b = synth.generate(3000, 9, 4, 3, seed=32)
+    pa = torch.from_numpy(a).pin_memory()
+    pb = torch.from_numpy(b).pin_memory()
+    with pk.Proclus(pa.numpy()) as h:
+        h.prefetch(pb.numpy())
+        ga = h.run(4, 3, seed=5)       # still dataset a
+        h.load(pb.numpy())              # waits for the prefetch, no second copy
+        gb = h.run(4, 3, seed=5)
+        h.prefetch(pa.numpy())
+        h.load(b)                       # a different pointer: plain copy wins
+        gb2 = h.run(4, 3, seed=5)
+    for g, data in ((ga, a), (gb, b), (gb2, b)):
+        o = orc.proclus(data, 4, 3, seed=5)
+        assert_parity(g, o, what="prefetch")
+
+
 def test_nonfinite_rejected(pk):
     data = np.random.default_rng(0).random((100, 4)).astype(np.float32)
     data[7, 1] = np.inf
