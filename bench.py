@@ -50,6 +50,8 @@ def workload_config(args, n_gpus):
                      "sd 5 on [0,100], 5% uniform noise, min-max normalised (P:374, P:386)",
         "l2": "256 MiB L2 flush written between timed steps",
         "parallelism": f"rows sharded over {n_gpus} GPU(s)" if n_gpus > 1 else "1 GPU",
+        "variant": {"fast": "GPU-FAST-PROCLUS", "plain": "GPU-PROCLUS (no caches, P:239)",
+                    "star": "GPU-FAST*-PROCLUS (P:215-219)"}[getattr(args, "variant", "fast")],
     }
 
 
@@ -211,6 +213,7 @@ def run_gpu(args):
     labels = torch.empty(hi - lo, dtype=torch.int32, device="cuda")
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device="cuda")
     common = dict(metric=metric, device=local, stream=stream.cuda_stream, world_size=world,
+                  variant={"fast": 0, "plain": 1, "star": 2}[args.variant],
                   rank=rank, n_global=n if world > 1 else 0, row_offset=lo if world > 1 else 0,
                   nccl_unique_id=uid)
     h = pk.Proclus(xdev, stats=(world > 1), **common)
@@ -305,7 +308,7 @@ def run_gpu(args):
     e2e = None
     if world == 1 and not args.no_e2e:
         pinned = torch.from_numpy(shard).pin_memory()
-        hh = pk.Proclus(pinned.numpy(), metric=metric, device=local)
+        hh = pk.Proclus(pinned.numpy(), metric=metric, device=local, variant=common["variant"])
         hlab = torch.empty(hi - lo, dtype=torch.int32).pin_memory()
         e_steps = max(3, min(args.steps, 20))
         for s in range(2):
@@ -504,6 +507,9 @@ def main():
     ap.add_argument("--seed0", type=int, default=1)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--variant", choices=["fast", "plain", "star"], default="fast",
+                    help="GPU-FAST-PROCLUS (default), GPU-PROCLUS without caches (P:239) "
+                         "or GPU-FAST*-PROCLUS (P:215-219)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: at least 3 warm-up steps

@@ -80,7 +80,23 @@ typedef struct {
   const void* nccl_unique_id;  /* 128-byte ncclUniqueId (world_size > 1)    */
   int32_t stats;           /* 1: time every kernel launch with CUDA events on
                               the handle's stream (see proclus_get_stats)   */
+  int32_t variant;         /* proclus_variant: which caches the iterative
+                              phase keeps; every variant returns the same
+                              clustering                     */
 } proclus_options;
+
+/* GPU-FAST-PROCLUS (default): the Dist row of every potential medoid is
+ * computed once and cached (#M x n fp32), with incremental
+ * locality bands and H (Theorems 3.1/3.2).
+ * GPU-PROCLUS: no caches; every iteration recomputes the k distance rows,
+ * the full L_i and X from scratch (the paper's ablation baseline).
+ * GPU-FAST*-PROCLUS: Dist rows and H are kept only for the current slots from
+ * the previous iteration (k x n fp32 instead of #M x n). */
+typedef enum {
+  PROCLUS_VARIANT_FAST = 0,
+  PROCLUS_VARIANT_PLAIN = 1,
+  PROCLUS_VARIANT_FAST_STAR = 2
+} proclus_variant;
 
 typedef struct {
   int32_t* labels;      /* [n] caller-allocated (host, or device if

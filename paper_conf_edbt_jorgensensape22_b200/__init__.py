@@ -23,6 +23,8 @@ LIB_PATH = _build.LIB
 
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, EINTERNAL = 0, -1, -2, -3, -4, -5
 METRIC_L2, METRIC_L1 = 0, 1
+# proclus_variant: GPU-FAST-PROCLUS, GPU-PROCLUS (no caches), GPU-FAST*-PROCLUS
+VARIANT_FAST, VARIANT_PLAIN, VARIANT_FAST_STAR = 0, 1, 2
 K_MAX = 32
 D_MAX = 256
 
@@ -38,7 +40,7 @@ class proclus_options(C.Structure):
                 ("data_on_device", C.c_int32), ("stream", C.c_void_p), ("trace", C.c_int32),
                 ("world_size", C.c_int32), ("rank", C.c_int32), ("n_global", C.c_int64),
                 ("row_offset", C.c_int64), ("nccl_unique_id", C.c_void_p),
-                ("stats", C.c_int32)]
+                ("stats", C.c_int32), ("variant", C.c_int32)]
 
 
 STAT_KINDS = ["pack", "gather", "greedy", "prepare", "locality", "assign", "cost",
@@ -213,7 +215,7 @@ class Proclus:
 
     def __init__(self, data, *, metric: int = METRIC_L2, device: int = -1,
                  max_iter: int = 0, trace: bool = False, stream: int | None = None,
-                 stats: bool = False,
+                 stats: bool = False, variant: int = VARIANT_FAST,
                  world_size: int = 1, rank: int = 0, n_global: int = 0,
                  row_offset: int = 0, nccl_unique_id: bytes | None = None):
         on_dev = hasattr(data, "is_cuda") and bool(data.is_cuda)
@@ -234,6 +236,7 @@ class Proclus:
         o.stream = stream
         o.trace = int(trace)
         o.stats = int(stats)
+        o.variant = int(variant)
         o.world_size = world_size
         o.rank = rank
         o.n_global = n_global

@@ -110,6 +110,7 @@ struct proclus_handle {
   int d = 0;
   int metric = 0, max_iter = 10000;
   bool data_on_device = false, trace = false, stats = false;
+  int variant = 0;  // proclus_variant
   int world = 1, rank = 0;
   ncclComm_t comm = nullptr;
   int num_sms = 148;
@@ -297,6 +298,8 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
     return fail(PROCLUS_EINVAL, "d must be in [2, %d] (got %d)", PROCLUS_D_MAX, d);
   if (o.metric != PROCLUS_METRIC_L2 && o.metric != PROCLUS_METRIC_L1)
     return fail(PROCLUS_EINVAL, "unknown metric %d", o.metric);
+  if (o.variant < PROCLUS_VARIANT_FAST || o.variant > PROCLUS_VARIANT_FAST_STAR)
+    return fail(PROCLUS_EINVAL, "unknown variant %d", o.variant);
   if (o.world_size < 1 || o.rank < 0 || o.rank >= o.world_size)
     return fail(PROCLUS_EINVAL, "bad world_size/rank");
   const int64_t n_total = o.n_global > 0 ? o.n_global : n;
@@ -322,6 +325,7 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
   h->data_on_device = o.data_on_device != 0;
   h->trace = o.trace != 0;
   h->stats = o.stats != 0;
+  h->variant = o.variant;
   h->world = o.world_size;
   h->rank = o.rank;
   proclus_status st = PROCLUS_OK;
@@ -542,8 +546,9 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   h->m_ksm = k_sm;
   h->m_A = A;
   h->m_B = B;
-  // new M: the Dist / H caches (keyed by M position) start empty
-  CK(h->dist.ensure((size_t)nM * h->n_pad));
+  // new M: the Dist / H caches (keyed by M position) start empty.  FAST*
+  // keeps k rows (allocated per setting), plain GPU-PROCLUS none.
+  if (h->variant == PROCLUS_VARIANT_FAST) CK(h->dist.ensure((size_t)nM * h->n_pad));
   CK(h->Hq.ensure((size_t)nM * d));
   CK(h->dprev.ensure((size_t)nM));
   CK(h->nL.ensure((size_t)nM));
@@ -632,6 +637,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   const PassShape ps = pass_shape(d, k, l, nM, h->num_sms);
   CK(configure_kernels(ps));
   CK(h->lab.ensure((size_t)2 * h->n_pad));
+  if (h->variant == PROCLUS_VARIANT_FAST_STAR) CK(h->dist.ensure((size_t)k * h->n_pad));
+  if (h->variant == PROCLUS_VARIANT_PLAIN) CK(h->dist.ensure(1));
   CK(h->med.ensure((size_t)KMAX * d));
   CK(h->X.ensure((size_t)KMAX * d));
   CK(h->Z.ensure((size_t)KMAX * d));
@@ -670,6 +677,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
     s.mbest[i] = pool[(size_t)i];
   }
   s.rng = it;
+  for (int i = 0; i < KMAX; ++i) s.cown[i] = -1;
   s.cost_best = INFINITY;
   s.cur_buf = 0;
   s.best_buf = 1;
@@ -721,6 +729,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.nchunks = (h->n + ps.P - 1) / ps.P;
   p.fuse_tail = h->world == 1 ? 1 : 0;
   p.cost1 = ps.cost1;
+  p.variant = h->variant;
   p.out_labels = h->out_labels.p;
   p.Delta = h->Delta.p;
   if (h->trace) {

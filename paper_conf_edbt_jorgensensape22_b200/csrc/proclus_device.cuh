@@ -21,7 +21,8 @@ constexpr int PAD_ALIGN = 1024;  // n_pad multiple; shard boundaries for invaria
 // (GPU-FAST-PROCLUS).  The band is (lo, hi]: Theorem 3.1 / eq 3.
 struct ActSlot {
   int slot;      // cluster slot i in MCur
-  int mpos;      // MIdx_i: position in M, row of Dist and H
+  int mpos;      // MIdx_i: position in M: the medoid's row of M
+  int key;       // cache row of Dist / H / |L| / delta': mpos (FAST) or slot (FAST*)
   int compute;   // 1: DistFound is false -> compute and store the Dist row
   int lam;       // lambda_i (eq 6): +1 grow, -1 shrink
   double lo, hi; // band (lo, hi]; lo = -inf on first use (L_i itself)
@@ -41,6 +42,7 @@ struct DevState {
   int n_act;
   ActSlot act[KMAX];
   int nD[KMAX];                 // |D_i|
+  int cown[KMAX];               // FAST*: M position cached in slot i's rows (-1: none)
   unsigned int ticket[4];       // last-block tickets of the pass kernels
   int err;
   double bytes_loc;             // algorithmic bytes of the locality passes
@@ -116,6 +118,7 @@ struct RunParams {
   long long nchunks;
   int fuse_tail;           // 1: last block finalises (single GPU)
   int cost1;               // 1: the cost pass sums per cluster (k_cost1), cells 0..k-1
+  int variant;             // proclus_variant: 0 FAST, 1 plain (no caches), 2 FAST*
   int use_cond;            // 1: running inside a graph while-node
   unsigned long long cond; // cudaGraphConditionalHandle
   TraceBufs tr;

@@ -1494,10 +1494,14 @@ __device__ void prepare_s(const RunParams& p, TailMem& T) {
     T.med[e] = (double)(cached ? T.mrow[r] : p.mrows[r]);
   }
   for (int i = tid; i < k; i += bd) {
+    // cache row of slot i: the M position (FAST), the slot if it still holds
+    // the same medoid as in the previous iteration (FAST*), none (plain)
     const int mp = S->mcur[i];
-    T.fnd[i] = cached ? T.fall[mp] : p.found[mp];
-    T.fnd[KMAX + i] = cached ? T.uall[mp] : p.used[mp];
-    T.fnd[2 * KMAX + i] = cached ? T.pall[mp] : p.dprev[mp];
+    const int key = p.variant == 2 ? i : mp;
+    const bool valid = p.variant == 0 || (p.variant == 2 && S->cown[i] == mp);
+    T.fnd[i] = valid ? (double)(cached ? T.fall[key] : p.found[key]) : 0.0;
+    T.fnd[KMAX + i] = valid ? (double)(cached ? T.uall[key] : p.used[key]) : 0.0;
+    T.fnd[2 * KMAX + i] = valid ? (cached ? T.pall[key] : p.dprev[key]) : 0.0;
   }
   __syncthreads();
   TST(T, 15);
@@ -1525,6 +1529,7 @@ __device__ void prepare_s(const RunParams& p, TailMem& T) {
       const double dp = T.fnd[2 * KMAX + i];
       a.slot = i;
       a.mpos = S->mcur[i];
+      a.key = p.variant == 2 ? i : a.mpos;
       a.compute = T.fnd[i] != 0.0 ? 0 : 1;
       a.lam = 1;
       on = true;
@@ -1580,38 +1585,44 @@ __device__ void tail_locality(const RunParams& p, TailMem& T) {
   const int na = S->n_act;
   for (int c = tid; c < kd; c += bd) {
     const int i = c / d, j = c - i * d;
-    const long long h = __ldcg(p.Hq + (long long)S->mcur[i] * d + j);
+    const int key = p.variant == 2 ? i : S->mcur[i];
+    const long long h = __ldcg(p.Hq + (long long)key * d + j);
     const long long v = c < na * d ? take_acc(p, c) : 0ll;
     Hs[c] = h;
     va[c] = v;
   }
   if (tid < k) {
-    const long long nl = __ldcg(p.nL + S->mcur[tid]);
+    const long long nl = __ldcg(p.nL + (p.variant == 2 ? tid : S->mcur[tid]));
     const long long v = tid < na ? take_cnt(p, tid) : 0ll;
     nL_s[tid] = nl;
     cnt_s[tid] = v;
   }
   for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
   if (tid == 0 && na > 0)  // byte model: data once + one Dist row per slot
-    S->bytes_loc += 4.0 * (double)p.n * (double)(d + na);
+    S->bytes_loc += 4.0 * (double)p.n * (double)(d + (p.variant == 1 ? 0 : na));
   __syncthreads();
   TST(T, 0);
   for (int c = tid; c < na * d; c += bd) {
     const int a = c / d, j = c - a * d;
     const ActSlot& A = S->act[a];
     const int e = A.slot * d + j;
-    const long long h = Hs[e] + (A.lam > 0 ? va[c] : -va[c]);
+    // first use of the cache row (lo = -inf): H = the sum over L_i itself
+    const long long h =
+        A.lo == -CUDART_INF ? va[c] : Hs[e] + (A.lam > 0 ? va[c] : -va[c]);
     Hs[e] = h;
-    p.Hq[(long long)A.mpos * d + j] = h;
+    p.Hq[(long long)A.key * d + j] = h;
   }
   if (tid < na) {
     const ActSlot& A = S->act[tid];
-    const long long nl = nL_s[A.slot] + (A.lam > 0 ? cnt_s[tid] : -cnt_s[tid]);
+    const long long nl = A.lo == -CUDART_INF
+                             ? cnt_s[tid]
+                             : nL_s[A.slot] + (A.lam > 0 ? cnt_s[tid] : -cnt_s[tid]);
     nL_s[A.slot] = nl;
-    p.nL[A.mpos] = nl;
-    p.dprev[A.mpos] = S->delta[A.slot];
-    p.used[A.mpos] = 1;
-    p.found[A.mpos] = 1;
+    p.nL[A.key] = nl;
+    p.dprev[A.key] = S->delta[A.slot];
+    p.used[A.key] = 1;
+    p.found[A.key] = p.variant == 1 ? 0 : 1;
+    if (p.variant == 2) S->cown[A.slot] = A.mpos;
   }
   __syncthreads();
   for (int c = tid; c < kd; c += bd) {
@@ -2076,7 +2087,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
     const unsigned b = __ballot_sync(0xffffffffu, cached);
     const int r = __popc(b & ((1u << a) - 1u));
     if (a < na) row_s[a] = cached ? (d + r) * R.ldr : -1;
-    if (cached) ex->src[r] = p.dist + (size_t)act_s[a].mpos * p.n_pad;
+    if (cached) ex->src[r] = p.dist + (size_t)act_s[a].key * p.n_pad;
     if (a == 0) ex->n = __popc(b);
   }
   // medoid rows at stride MS (zero padded to DR for float4 loads)
@@ -2147,7 +2158,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
                 s = approx_full(xs + q, LD, m, d, metric);
               }
               f = s;
-              p.dist[(long long)act_s[a].mpos * p.n_pad + gp] = f;
+              if (p.variant != 1) p.dist[(long long)act_s[a].key * p.n_pad + gp] = f;
             } else {
               f = xs[rs + q];
             }

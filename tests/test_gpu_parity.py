@@ -21,8 +21,8 @@ def pk():
 
 
 def run_both(pk, orc, data, k, l, *, A=100, B=10, minDev=0.7, itrPat=5, seed=1,
-             metric=0, trace=True):
-    with pk.Proclus(data, metric=metric, trace=trace) as h:
+             metric=0, trace=True, variant=0):
+    with pk.Proclus(data, metric=metric, trace=trace, variant=variant) as h:
         g = h.run(k, l, A, B, minDev, itrPat, seed)
         gt = h.trace() if trace else None
     o = orc.proclus(data, k, l, A, B, minDev, itrPat, seed, metric=metric, trace=trace)
@@ -235,5 +235,53 @@ def test_full_size_configs(pk, orc, name, seed):
     data, cfg = synth.config_data(name, seed=seed)
     g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
     note = assert_parity(g, o, gt, ot, what=name)
+    if note:
+        pytest.skip(note)
+
+
+# ------------------------------------------------ variants
+# GPU-PROCLUS (no caches) and GPU-FAST*-PROCLUS (slot caches from the
+# previous iteration only) must reach the same clustering as plain
+# PROCLUS -- the oracle -- on the same draws.
+@pytest.mark.parametrize("variant", [1, 2])
+@pytest.mark.parametrize("seed", range(1, 9))
+def test_variants_C1(pk, orc, variant, seed):
+    data, cfg = synth.config_data("C1", seed=seed)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed, variant=variant)
+    note = assert_parity(g, o, gt, ot, what=f"variant {variant} C1 seed {seed}")
+    if note:
+        pytest.skip(note)
+
+
+@pytest.mark.parametrize("variant", [1, 2])
+@pytest.mark.parametrize("shape", [(3001, 16, 6, 4, 30, 6), (4097, 33, 8, 6, 20, 5),
+                                   (1500, 100, 10, 10, 20, 5)])
+def test_variants_shapes(pk, orc, variant, shape):
+    n, d, k, l, A, B = shape
+    data = synth.generate(n, d, max(2, k // 2), max(1, d // 3), seed=n)
+    g, gt, o, ot = run_both(pk, orc, data, k, l, A=A, B=B, seed=3, variant=variant)
+    note = assert_parity(g, o, gt, ot, what=f"variant {variant} shape {shape}")
+    if note:
+        pytest.skip(note)
+
+
+@pytest.mark.parametrize("variant", [1, 2])
+def test_variants_C2_and_multi(pk, orc, variant):
+    data, cfg = synth.config_data("C2", seed=1)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=1, variant=variant)
+    assert_parity(g, o, gt, ot, what=f"variant {variant} C2")
+    small = synth.generate(6000, 10, 5, 3, seed=12)
+    with pk.Proclus(small, variant=variant) as h:
+        got = h.run_multi([3, 5], [2, 4], seed=7, reuse_level=2)
+    want = orc.proclus_multi(small, [3, 5], [2, 4], seed=7, reuse_level=2)
+    for i, (gg, oo) in enumerate(zip(got, want)):
+        assert_parity(gg, oo, what=f"variant {variant} multi setting {i}")
+
+
+@pytest.mark.parametrize("variant", [1, 2])
+def test_variants_full_size_C3(pk, orc, variant):
+    data, cfg = synth.config_data("C3", seed=1)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=1, variant=variant)
+    note = assert_parity(g, o, gt, ot, what=f"variant {variant} C3")
     if note:
         pytest.skip(note)
