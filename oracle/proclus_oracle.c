@@ -565,7 +565,8 @@ static void gather_rows(const float* data, int32_t d, const int64_t* ids,
 static int run_core(const float* data, int64_t n, int32_t d,
                     const int64_t* Mid /* point ids of M, nM */, int64_t nM,
                     const oracle_params* prm, uint64_t it_state,
-                    oracle_result* out, oracle_trace* tr) {
+                    oracle_result* out, oracle_trace* tr,
+                    const int64_t* warm, int32_t nwarm, int64_t* mbest_out) {
   const int32_t k = prm->k, l = prm->l, metric = prm->metric;
   const int32_t max_iter = prm->max_iter > 0 ? prm->max_iter : 10000;
   int32_t i, j, itr = 0, iterations = 0;
@@ -606,14 +607,46 @@ static int run_core(const float* data, int64_t n, int32_t d,
     goto done;
   }
 
-  /* O5 [R12]: MCur = k distinct positions of M (partial Fisher-Yates). */
-  for (t = 0; t < nM; ++t) pool[t] = t;
-  for (i = 0; i < k; ++i) {
-    int64_t r = i + (int64_t)oracle_uniform(&st, (uint64_t)(nM - i));
-    int64_t tmp = pool[i];
-    pool[i] = pool[r];
-    pool[r] = tmp;
-    MCur[i] = pool[i];
+  if (warm && nwarm > 0) {
+    /* Multi-param level 3 [R21]: MCur is a random subset of the
+     * previous setting's MBest: partial Fisher-Yates over MBest_prev in slot
+     * order for the first min(k, |MBest_prev|) slots; if k is larger, the
+     * remaining slots by partial Fisher-Yates over the ascending positions of
+     * M not in MBest_prev.  All draws from stream IT, in slot order. */
+    const int32_t m = k < nwarm ? k : nwarm;
+    int64_t np2 = 0;
+    for (t = 0; t < nwarm; ++t) pool[t] = warm[t];
+    for (i = 0; i < m; ++i) {
+      int64_t r = i + (int64_t)oracle_uniform(&st, (uint64_t)(nwarm - i));
+      int64_t tmp = pool[i];
+      pool[i] = pool[r];
+      pool[r] = tmp;
+      MCur[i] = pool[i];
+    }
+    if (k > nwarm) {
+      for (t = 0; t < nM; ++t) inpool[t] = 1;
+      for (t = 0; t < nwarm; ++t) inpool[warm[t]] = 0;
+      for (t = 0; t < nM; ++t)
+        if (inpool[t]) pool[np2++] = t;
+      for (i = nwarm; i < k; ++i) {
+        const int64_t u = i - nwarm;
+        int64_t r = u + (int64_t)oracle_uniform(&st, (uint64_t)(np2 - u));
+        int64_t tmp = pool[u];
+        pool[u] = pool[r];
+        pool[r] = tmp;
+        MCur[i] = pool[u];
+      }
+    }
+  } else {
+    /* O5 [R12]: MCur = k distinct positions of M (partial Fisher-Yates). */
+    for (t = 0; t < nM; ++t) pool[t] = t;
+    for (i = 0; i < k; ++i) {
+      int64_t r = i + (int64_t)oracle_uniform(&st, (uint64_t)(nM - i));
+      int64_t tmp = pool[i];
+      pool[i] = pool[r];
+      pool[r] = tmp;
+      MCur[i] = pool[i];
+    }
   }
   for (i = 0; i < k; ++i) MBest[i] = MCur[i];
   if (tr) tr->count = 0;
@@ -715,6 +748,8 @@ static int run_core(const float* data, int64_t n, int32_t d,
   memcpy(out->dims, dmask, (size_t)k * d);
   out->cost = costBest;
   out->iterations = iterations;
+  if (mbest_out)
+    for (i = 0; i < k; ++i) mbest_out[i] = MBest[i];
   (void)j;
 
 done:
@@ -787,7 +822,7 @@ int oracle_proclus(const float* data, int64_t n, int32_t d,
   out->nS = nS;
   out->nM = nM;
   rc = run_core(data, n, d, Mid, nM, prm,
-                oracle_stream_it(prm->seed, prm->k, prm->l), out, trace);
+                oracle_stream_it(prm->seed, prm->k, prm->l), out, trace, NULL, 0, NULL);
   free(Mid);
   return rc;
 }
@@ -800,7 +835,7 @@ int oracle_proclus_multi(const float* data, int64_t n, int32_t d,
   int64_t nS = 0, nM = 0, *Mid = NULL;
   int rc = ORC_OK;
   oracle_params p = *base;
-  if (nk < 1 || nl < 1 || (reuse_level != 1 && reuse_level != 2)) return ORC_EINVAL;
+  if (nk < 1 || nl < 1 || reuse_level < 1 || reuse_level > 3) return ORC_EINVAL;
   for (a = 0; a < nk; ++a) {
     if (ks[a] > kmax) kmax = ks[a];
     for (b = 0; b < nl; ++b) {
@@ -820,19 +855,32 @@ int oracle_proclus_multi(const float* data, int64_t n, int32_t d,
       }
     return ORC_OK;
   }
-  /* Level 2: greedy once for the largest k, shared M. */
+  /* Level 2: greedy once for the largest k, shared M.  Level 3
+   * [R21]: every setting after the first starts from a random subset
+   * of the previous setting's MBest (grid in caller order). */
   p.k = kmax;
   rc = init_phase(data, n, d, kmax, &p, &nS, &nM, &Mid);
   if (rc != ORC_OK) return rc;
-  for (a = 0; a < nk && rc == ORC_OK; ++a)
-    for (b = 0; b < nl && rc == ORC_OK; ++b) {
-      p.k = ks[a];
-      p.l = ls[b];
-      outs[a * nl + b].nS = nS;
-      outs[a * nl + b].nM = nM;
-      rc = run_core(data, n, d, Mid, nM, &p,
-                    oracle_stream_it(p.seed, p.k, p.l), &outs[a * nl + b], NULL);
-    }
+  {
+    int64_t* warm = (int64_t*)malloc(sizeof(int64_t) * (size_t)kmax);
+    int64_t* next = (int64_t*)malloc(sizeof(int64_t) * (size_t)kmax);
+    int32_t nwarm = 0;
+    if (!warm || !next) rc = ORC_ENOMEM;
+    for (a = 0; a < nk && rc == ORC_OK; ++a)
+      for (b = 0; b < nl && rc == ORC_OK; ++b) {
+        p.k = ks[a];
+        p.l = ls[b];
+        outs[a * nl + b].nS = nS;
+        outs[a * nl + b].nM = nM;
+        rc = run_core(data, n, d, Mid, nM, &p, oracle_stream_it(p.seed, p.k, p.l),
+                      &outs[a * nl + b], NULL, reuse_level == 3 ? warm : NULL,
+                      reuse_level == 3 ? nwarm : 0, next);
+        memcpy(warm, next, sizeof(int64_t) * (size_t)p.k);
+        nwarm = p.k;
+      }
+    free(warm);
+    free(next);
+  }
   free(Mid);
   return rc;
 }

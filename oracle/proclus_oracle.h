@@ -124,8 +124,11 @@ int oracle_proclus(const float* data, int64_t n, int32_t d,
                    oracle_trace* trace);
 /* Multi-parameter. reuse_level 1: every setting == an
  * independent oracle_proclus(k,l,seed). reuse_level 2: S and M drawn once
- * for k_max (stream SM keyed by k_max) and shared by every setting. outs is
- * [nk*nl], k outer, l inner; each outs[i] has its own arrays. */
+ * for k_max (stream SM keyed by k_max) and shared by every setting.
+ * reuse_level 3 (reading R21): level 2, and every setting after the
+ * first draws its initial MCur as a random subset of the previous setting's
+ * MBest (topped up from M \ MBest_prev when k grows). outs is [nk*nl], k
+ * outer, l inner; each outs[i] has its own arrays. */
 int oracle_proclus_multi(const float* data, int64_t n, int32_t d,
                          const int32_t* ks, int32_t nk, const int32_t* ls,
                          int32_t nl, const oracle_params* base,

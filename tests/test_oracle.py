@@ -454,3 +454,37 @@ def test_multi_levels(orc):
     assert all(r.nM == 40 and r.nS == 400 for r in m2)
     for r, (k, l) in zip(m2, itertools.product(ks, ls)):
         assert r.dims.sum() == k * l
+
+
+def test_multi_level3_warm_start(orc):
+    """P:213 level 3 [R21]: the first setting is level 2's; a repeated (k, l)
+    starts from a permutation of the previous MBest, so its costBest cannot
+    exceed the previous one (slot order changes only the rounding of eq 2).
+    Level 2 repeats the first run exactly (same stream IT); level 3 must not
+    (its start differs) for some seed."""
+    data = synth.generate(3000, 8, 4, 3, seed=21)
+    differs = 0
+    for seed in range(1, 9):
+        m2 = orc.proclus_multi(data, [4, 4], [3], seed=seed, reuse_level=2)
+        m3 = orc.proclus_multi(data, [4, 4], [3], seed=seed, reuse_level=3)
+        assert np.array_equal(m3[0].labels, m2[0].labels) and m3[0].cost == m2[0].cost
+        assert m3[1].cost <= m3[0].cost * (1 + 1e-12)
+        assert np.array_equal(m2[1].labels, m2[0].labels) and m2[1].cost == m2[0].cost
+        differs += m3[1].iterations != m2[1].iterations or not np.array_equal(
+            m3[1].medoids, m2[1].medoids)
+        for r in m3:
+            assert r.dims.sum() == 4 * 3 and (r.dims.sum(axis=1) >= 2).all()
+            assert len(set(r.medoids.tolist())) == 4
+    assert differs > 0
+
+
+def test_multi_level3_grid_shapes(orc):
+    """Level 3 over a grid where k grows and shrinks (top-up from M \ MBest
+    and subsets of MBest): invariants of every setting."""
+    data = synth.generate(2500, 9, 5, 3, seed=22)
+    ks, ls = [3, 5, 2], [2, 4]
+    m3 = orc.proclus_multi(data, ks, ls, seed=3, reuse_level=3)
+    for r, (k, l) in zip(m3, itertools.product(ks, ls)):
+        assert r.dims.sum() == k * l and (r.dims.sum(axis=1) >= 2).all()
+        assert len(set(r.medoids.tolist())) == k
+        assert ((r.labels >= -1) & (r.labels < k)).all()
