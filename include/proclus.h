@@ -194,7 +194,13 @@ PROCLUS_API proclus_status proclus_run(proclus_handle* h, int32_t k, int32_t l, 
  *   share M, i.e. the same k).
  * reuse_level 2: S and M are drawn once for k_max (greedy once) and
  *   Dist, H, delta', |L| are reused across the whole grid ("multi-param 2").
- * EINVAL: reuse_level not in {1,2}, empty grid, any invalid (k, l). */
+ * reuse_level 3: level 2, and every setting after the first starts from a
+ *   random subset of the previous setting's MBest ("multi-param 3";
+ *   reading R21: partial Fisher-Yates over MBest_prev in slot order, topped
+ *   up from the ascending positions of M \ MBest_prev when k grows; stream
+ *   IT of the setting).  This heuristic changes the results: settings are
+ *   sequential in caller order.
+ * EINVAL: reuse_level not in {1,2,3}, empty grid, any invalid (k, l). */
 PROCLUS_API proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks,
                                  int32_t nk, const int32_t* ls, int32_t nl,
                                  int32_t A, int32_t B, double minDev,

@@ -631,7 +631,8 @@ static proclus_status build_graph(proclus_handle* h, RunParams p, const PassShap
 }
 
 static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev, int itrPat,
-                                  uint64_t seed, proclus_result* out) {
+                                  uint64_t seed, proclus_result* out,
+                                  const std::vector<int>* warm = nullptr) {
   const int d = h->d;
   const int nM = (int)h->nM;
   const PassShape ps = pass_shape(d, k, l, nM, h->num_sms);
@@ -667,14 +668,40 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   // initial MCur: k distinct positions of M (partial Fisher-Yates, stream IT)
   uint64_t it = stream_it(seed, k, l);
   std::vector<int> pool((size_t)nM);
-  for (int t = 0; t < nM; ++t) pool[(size_t)t] = t;
   DevState& s = *h->h_st;
   memset(&s, 0, sizeof(s));
-  for (int i = 0; i < k; ++i) {
-    int r = i + (int)sm_uniform(&it, (uint64_t)(nM - i));
-    std::swap(pool[(size_t)i], pool[(size_t)r]);
-    s.mcur[i] = pool[(size_t)i];
-    s.mbest[i] = pool[(size_t)i];
+  if (warm && !warm->empty()) {
+    // multi-param level 3 (reading R21): a random subset of the
+    // previous setting's MBest (slot order), topped up from M \ MBest_prev
+    const int nw = (int)warm->size(), m = std::min(k, nw);
+    std::vector<int> wp(*warm);
+    for (int i = 0; i < m; ++i) {
+      int r = i + (int)sm_uniform(&it, (uint64_t)(nw - i));
+      std::swap(wp[(size_t)i], wp[(size_t)r]);
+      s.mcur[i] = wp[(size_t)i];
+    }
+    if (k > nw) {
+      std::vector<char> in((size_t)nM, 1);
+      for (int v : *warm) in[(size_t)v] = 0;
+      int np2 = 0;
+      for (int t = 0; t < nM; ++t)
+        if (in[(size_t)t]) pool[(size_t)np2++] = t;
+      for (int i = nw; i < k; ++i) {
+        const int u = i - nw;
+        int r = u + (int)sm_uniform(&it, (uint64_t)(np2 - u));
+        std::swap(pool[(size_t)u], pool[(size_t)r]);
+        s.mcur[i] = pool[(size_t)u];
+      }
+    }
+    for (int i = 0; i < k; ++i) s.mbest[i] = s.mcur[i];
+  } else {
+    for (int t = 0; t < nM; ++t) pool[(size_t)t] = t;
+    for (int i = 0; i < k; ++i) {
+      int r = i + (int)sm_uniform(&it, (uint64_t)(nM - i));
+      std::swap(pool[(size_t)i], pool[(size_t)r]);
+      s.mcur[i] = pool[(size_t)i];
+      s.mbest[i] = pool[(size_t)i];
+    }
   }
   s.rng = it;
   for (int i = 0; i < KMAX; ++i) s.cown[i] = -1;
@@ -869,8 +896,8 @@ proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks, int32_t n
                                  int32_t reuse_level, proclus_result* outs) {
   if (!h || !ks || !ls || !outs) return fail(PROCLUS_EINVAL, "NULL argument");
   if (nk < 1 || nl < 1) return fail(PROCLUS_EINVAL, "empty parameter grid");
-  if (reuse_level != 1 && reuse_level != 2)
-    return fail(PROCLUS_EINVAL, "reuse_level must be 1 or 2 (3 is not implemented)");
+  if (reuse_level < 1 || reuse_level > 3)
+    return fail(PROCLUS_EINVAL, "reuse_level must be 1, 2 or 3");
   int kmax = 0;
   for (int a = 0; a < nk; ++a) {
     kmax = std::max(kmax, ks[a]);
@@ -883,11 +910,14 @@ proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks, int32_t n
   }
   TRY(set_device(h));
   reset_stats(h);
-  if (reuse_level == 2) TRY(init_phase(h, kmax, A, B, seed));
+  if (reuse_level >= 2) TRY(init_phase(h, kmax, A, B, seed));
+  std::vector<int> warm;  // level 3: MBest (positions in M) of the previous setting
   for (int a = 0; a < nk; ++a)
     for (int b = 0; b < nl; ++b) {
       if (reuse_level == 1) TRY(init_phase(h, ks[a], A, B, seed));
-      TRY(run_setting(h, ks[a], ls[b], minDev, itrPat, seed, &outs[a * nl + b]));
+      TRY(run_setting(h, ks[a], ls[b], minDev, itrPat, seed, &outs[a * nl + b],
+                      reuse_level == 3 ? &warm : nullptr));
+      if (reuse_level == 3) warm.assign(h->h_st->mbest, h->h_st->mbest + ks[a]);
     }
   return PROCLUS_OK;
 }

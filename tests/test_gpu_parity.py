@@ -158,6 +158,19 @@ def test_load_replaces_data(pk, orc):
     assert_parity(g, orc.proclus(d2, 5, 3, seed=1), what="after load")
 
 
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_run_multi_level3_grids(pk, orc, seed):
+    """Level 3 over a grid where k grows and shrinks, and a repeated
+    setting (warm start from a permutation of MBest)."""
+    data = synth.generate(5000, 9, 5, 3, seed=40 + seed)
+    for ks, ls in (([3, 5, 2], [2, 4]), ([4, 4], [3])):
+        with pk.Proclus(data) as h:
+            got = h.run_multi(ks, ls, seed=seed, reuse_level=3)
+        want = orc.proclus_multi(data, ks, ls, seed=seed, reuse_level=3)
+        for i, (g, o) in enumerate(zip(got, want)):
+            assert_parity(g, o, what=f"level 3 {ks}x{ls} setting {i}")
+
+
 def test_prefetch_overlaps_next_dataset(pk, orc):
     """proclus_prefetch stages the next dataset while the current one is
     clustered; load() of the same pointer then swaps it in (P:87 per step)."""
@@ -219,7 +232,7 @@ def test_device_resident_io(pk, orc):
 def test_run_multi_levels(pk, orc):
     data = synth.generate(6000, 10, 5, 3, seed=12)
     ks, ls = [3, 5], [2, 4]
-    for level in (1, 2):
+    for level in (1, 2, 3):
         with pk.Proclus(data) as h:
             got = h.run_multi(ks, ls, seed=7, reuse_level=level)
         want = orc.proclus_multi(data, ks, ls, seed=7, reuse_level=level)
