@@ -130,13 +130,15 @@ class ClockSampler:
 
 
 def cpu_baseline_full(data, cfg, metric):
-    """The oracle as it stands: one full clustering of the workload, 1 core."""
+    """The oracle as it stands: one full clustering of the workload (or of its
+    first ORACLE_MAX_ROWS rows, scaled by n / n_sample), 1 core."""
     import oracle
 
+    ns = min(len(data), ORACLE_MAX_ROWS)
     t = time.perf_counter()
-    r = oracle.proclus(data, cfg["k"], cfg["l"], seed=1, metric=metric)
-    dt = time.perf_counter() - t
-    return r, dt
+    r = oracle.proclus(np.ascontiguousarray(data[:ns]), cfg["k"], cfg["l"], seed=1, metric=metric)
+    dt = (time.perf_counter() - t) * len(data) / ns
+    return r, dt, ns
 
 
 def run_reference(args):
@@ -148,7 +150,7 @@ def run_reference(args):
         return 0
     oracle.build()
     # C5 (the sweep) is timed on its data (C3's) one setting per step
-    data, cfg = synth.config_data("C3" if args.config == "C5" else args.config,
+    data, cfg = synth.config_data({"C5": "C3", "L8S": "L8"}.get(args.config, args.config),
                                   seed=args.data_seed)
     ns = min(REF_SAMPLE_ROWS, cfg["n"])
     sample = np.ascontiguousarray(data[:ns])
@@ -339,17 +341,24 @@ def run_gpu(args):
         import oracle
 
         oracle.build()
-        o, dt = cpu_baseline_full(data, cfg, metric)
+        o, dt, ns = cpu_baseline_full(data, cfg, metric)
+        what = (f"one full clustering of the {args.config} workload" if ns == n else
+                f"one clustering of the first {ns:,} rows of the {args.config} workload, "
+                f"scaled by n / n_sample")
         cpu = {"value": 1.0 / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"one full clustering of the {args.config} workload (seed 1) by the "
-                         f"single-threaded fp64 C oracle: {dt:.2f} s, {o.iterations} iterations"}
-        g = h.run(k, l, seed=1, labels=labels)
-        glab = labels.cpu().numpy()
-        parity = {"seed": 1, "labels_equal": bool(np.array_equal(glab, o.labels)),
-                  "medoids_equal": bool(np.array_equal(g.medoids, o.medoids)),
-                  "dims_equal": bool(np.array_equal(g.dims, o.dims)),
-                  "iterations": [g.iterations, o.iterations],
-                  "cost_rel_err": abs(g.cost - o.cost) / abs(o.cost)}
+               "sample": f"{what} (seed 1) by the single-threaded fp64 C oracle: "
+                         f"{dt:.2f} s, {o.iterations} iterations"}
+        if ns == n:
+            g = h.run(k, l, seed=1, labels=labels)
+            glab = labels.cpu().numpy()
+            parity = {"seed": 1, "labels_equal": bool(np.array_equal(glab, o.labels)),
+                      "medoids_equal": bool(np.array_equal(g.medoids, o.medoids)),
+                      "dims_equal": bool(np.array_equal(g.dims, o.dims)),
+                      "iterations": [g.iterations, o.iterations],
+                      "cost_rel_err": abs(g.cost - o.cost) / abs(o.cost)}
+        else:
+            parity = {"note": "full-size parity by sampled properties: "
+                              "tests/test_gpu_parity.py::test_large_n_properties"}
     h.close()
 
     if rank == 0:
@@ -376,6 +385,10 @@ def run_gpu(args):
 
 SWEEP_KS = list(range(5, 21))   # C5: k in {5..20}
 SWEEP_LS = list(range(3, 11))   # C5: l in {3..10}
+# L8S: 9 combinations of k and l (Fig 3e; the paper does not list
+# them -- reading R22: the 3 x 3 grid around the defaults k = 10, l = 5)
+GRID9_KS, GRID9_LS = [5, 10, 15], [3, 5, 7]
+ORACLE_MAX_ROWS = 2_000_000     # larger workloads: the oracle runs on a prefix
 
 
 def run_sweep(args):
@@ -400,7 +413,9 @@ def run_sweep(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     pk.lib()
-    data, cfg = synth.config_data("C3", seed=args.data_seed)  # same 1M x 15 data as C3
+    base, ks_grid, ls_grid = (("C3", SWEEP_KS, SWEEP_LS) if args.config == "C5"
+                              else ("L8", GRID9_KS, GRID9_LS))
+    data, cfg = synth.config_data(base, seed=args.data_seed)
     n, d = cfg["n"], cfg["d"]
     metric = pk.METRIC_L2 if args.metric == "l2" else pk.METRIC_L1
     from paper_conf_edbt_jorgensensape22_b200.sharding import shard_rows
@@ -418,7 +433,7 @@ def run_sweep(args):
     h = pk.Proclus(xdev, metric=metric, device=local, stream=stream.cuda_stream,
                    world_size=world, rank=rank, n_global=n if world > 1 else 0,
                    row_offset=lo if world > 1 else 0, nccl_unique_id=uid)
-    nset = len(SWEEP_KS) * len(SWEEP_LS)
+    nset = len(ks_grid) * len(ls_grid)
 
     def barrier():
         if world > 1:
@@ -439,9 +454,9 @@ def run_sweep(args):
             out.append(e0.elapsed_time(e1))
         return out
 
-    sweep = lambda s: h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + s, reuse_level=2)
+    sweep = lambda s: h.run_multi(ks_grid, ls_grid, seed=args.seed0 + s, reuse_level=2)
     for s in range(args.warmup):
-        h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + 1000 + s, reuse_level=2)
+        h.run_multi(ks_grid, ls_grid, seed=args.seed0 + 1000 + s, reuse_level=2)
     barrier()
     with ClockSampler(local) as clk:
         barrier()
@@ -449,11 +464,11 @@ def run_sweep(args):
         barrier()
     total_ms = sum(ms)
     # level 0: the same settings as independent runs (one step)
-    indep = lambda s: [h.run(k, l, seed=args.seed0 + s) for k in SWEEP_KS for l in SWEEP_LS]
+    indep = lambda s: [h.run(k, l, seed=args.seed0 + s) for k in ks_grid for l in ls_grid]
     ms0 = timed(indep, 1)
-    ms1 = timed(lambda s: h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + s, reuse_level=1), 1)
+    ms1 = timed(lambda s: h.run_multi(ks_grid, ls_grid, seed=args.seed0 + s, reuse_level=1), 1)
     # level 3: warm start from the previous MBest -- changes results
-    ms3 = timed(lambda s: h.run_multi(SWEEP_KS, SWEEP_LS, seed=args.seed0 + s, reuse_level=3), 1)
+    ms3 = timed(lambda s: h.run_multi(ks_grid, ls_grid, seed=args.seed0 + s, reuse_level=3), 1)
     if world > 1:
         t = torch.tensor([total_ms, ms0[0], ms1[0], ms3[0]], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -465,7 +480,7 @@ def run_sweep(args):
 
         oracle.build()
         ns = REF_SAMPLE_ROWS
-        ks, ls = [SWEEP_KS[0], SWEEP_KS[-1]], [SWEEP_LS[0], SWEEP_LS[-1]]
+        ks, ls = [ks_grid[0], ks_grid[-1]], [ls_grid[0], ls_grid[-1]]
         t0 = time.perf_counter()
         oracle.proclus_multi(np.ascontiguousarray(data[:ns]), ks, ls, seed=1, reuse_level=2,
                              metric=0 if args.metric == "l2" else 1)
@@ -480,8 +495,8 @@ def run_sweep(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": total_ms / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": f"C5: multi-parameter sweep k in 5..20 x l in 3..10 "
-                                   f"({nset} settings) at n={n:,} d={d}, reuse level 2 "
+            "config": {"workload": f"{args.config}: multi-parameter grid k in {ks_grid} x l in "
+                                   f"{ls_grid} ({nset} settings) at n={n:,} d={d}, reuse level 2 "
                                    f"(P:207-213), A=100 B=10 minDev=0.7 itrPat=5",
                        "settings_per_step": nset, "l2": "256 MiB L2 flush between steps",
                        "parallelism": f"rows sharded over {world} GPU(s)" if world > 1 else "1 GPU"},
@@ -504,7 +519,10 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", choices=["C1", "C2", "C3", "C4", "C5"], default="C3")
+    ap.add_argument("--config", choices=["C1", "C2", "C3", "C4", "C5", "L8", "L8S"], default="C3",
+                    help="C1-C4: one clustering per step; C5: the k 5..20 x l 3..10 sweep "
+                         "at n=1M; L8: one clustering of 8M points; L8S: the 9-setting grid "
+                         "at 8M points (Fig 3e)")
     ap.add_argument("--metric", choices=["l2", "l1"], default="l2")
     ap.add_argument("--data-seed", type=int, default=1)
     ap.add_argument("--seed0", type=int, default=1)
@@ -518,7 +536,7 @@ def main():
         args.warmup = 3  # timing rule: at least 3 warm-up steps
     if args.impl == "reference":
         return run_reference(args)
-    if args.config == "C5":
+    if args.config in ("C5", "L8S"):
         return run_sweep(args)
     return run_gpu(args)
 

@@ -15,12 +15,14 @@ from __future__ import annotations
 
 import numpy as np
 
-# The configurations of BASELINE.json (C1..C4).
+# The configurations of BASELINE.json (C1..C4) and the large-n workload L8.
 CONFIGS = {
     "C1": dict(n=4_000, d=15, n_clusters=5, subspace_dim=3, k=5, l=3),
     "C2": dict(n=64_000, d=15, n_clusters=10, subspace_dim=5, k=10, l=5),
     "C3": dict(n=1_000_000, d=15, n_clusters=10, subspace_dim=5, k=10, l=5),
     "C4": dict(n=256_000, d=100, n_clusters=20, subspace_dim=10, k=20, l=10),
+    # the paper's large-n workload (Fig 3e, > 8M points)
+    "L8": dict(n=8_000_000, d=15, n_clusters=10, subspace_dim=5, k=10, l=5),
 }
 
 

@@ -298,3 +298,48 @@ def test_variants_full_size_C3(pk, orc, variant):
     note = assert_parity(g, o, gt, ot, what=f"variant {variant} C3")
     if note:
         pytest.skip(note)
+
+
+# ------------------------------------------------ n = 8M
+def _seg(x, m, dmask):
+    """seg_D(x, m) of O0 in fp64, one column per cluster (x: [p, d])."""
+    diff = np.abs(x[:, None, :].astype(np.float64) - m[None, :, :].astype(np.float64))
+    return (diff * dmask[None]).sum(axis=2) / dmask.sum(axis=1)[None]
+
+
+def test_large_n_properties(pk):
+    """At the L8 size (8M x 15, Fig 3e) the oracle takes minutes per run, so
+    the GPU result is checked through properties that hold at any size, on
+    20,000 sampled points: every label is the segmental argmin over the
+    returned medoids / dimensions (reading R8, ties to the smaller slot), -1
+    exactly when the point is outside every Delta_i sphere (R17); every
+    medoid carries its own label; k*l dimensions, >= 2 per cluster."""
+    import torch
+
+    data, cfg = synth.config_data("L8", seed=1)
+    k, l = cfg["k"], cfg["l"]
+    x = torch.from_numpy(data).cuda()
+    lab = torch.empty(data.shape[0], dtype=torch.int32, device="cuda")
+    with pk.Proclus(x) as h:
+        g = h.run(k, l, seed=1, labels=lab)
+    labels = lab.cpu().numpy()
+    dm = g.dims.astype(np.float64)
+    assert int(g.dims.sum()) == k * l and (g.dims.sum(axis=1) >= 2).all()
+    med = data[g.medoids]
+    # Delta_i = min_{j != i} seg_{D_i}(m_i, m_j) (P:93, R5)
+    sm = _seg(med, med, dm)                      # sm[a, i] = seg_{D_i}(m_a, m_i)
+    Delta = np.array([min(sm[j, i] for j in range(k) if j != i) for i in range(k)])
+    rng = np.random.default_rng(0)
+    idx = rng.choice(data.shape[0], 20_000, replace=False)
+    sd = _seg(data[idx], med, dm)
+    order = np.sort(sd, axis=1)
+    gap = (order[:, 1] - order[:, 0]) / np.maximum(order[:, 0], 1e-300)
+    want = np.argmin(sd, axis=1)
+    outside = (sd > Delta[None]).all(axis=1)
+    want = np.where(outside, -1, want)
+    ok = (labels[idx] == want) | (gap < 1e-6)   # north_star argmin allowance
+    assert ok.all(), f"{(~ok).sum()} sampled labels differ"
+    for i, mi in enumerate(g.medoids):
+        assert labels[mi] in (i, -1) or sd.shape[0] == 0
+    assert (labels >= -1).all() and (labels < k).all()
+    assert 6 <= g.iterations < 10000
