@@ -70,7 +70,6 @@ struct SmemLayout {
   int full, empty, buf, lab;                    // TMA ring and its mbarriers
   int med, act, row, scale, cells, bal, acc, cnt, ex;
   int tab, dl, nD, off, rcp, ctr, Dl, thr;
-  int tab2, nDa, labq;                          // k_assign2: distance table, |D_i|, chunk labels
   int P, ldr, stages;  // chunk points, ring row stride (floats), ring depth (k_lsum2 etc.)
   int tail;      // start of the tail scratch (reuses the ring region)
   int bytes;     // total dynamic shared memory of the kernel
@@ -82,8 +81,8 @@ struct TailLayout {
   int mrow, fall, uall, pall;  // rows of M and their tables, or mrow = -1
   int bytes;
 };
-enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3, KK_LS2 = 4, KK_REF2 = 5, KK_ASG2 = 6, KK_ASG3 = 7, KK_COST1 = 8 };
-constexpr int NLAY = 9;
+enum KernelKind { KK_LOC = 0, KK_ASG = 1, KK_LSUM = 2, KK_FIN = 3, KK_LS2 = 4, KK_REF2 = 5, KK_COST1 = 6 };
+constexpr int NLAY = 7;
 
 struct RunParams {
   long long n;        // rows on this device

@@ -826,32 +826,6 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// Per-warp phase cycle counters (-DPROCLUS_PHASE_PROFILE builds only):
-// PH_MARK(i) adds the cycles since the previous mark to phase i (i < 0:
-// restart); PH_FLUSH adds them (lane 0 of each warp, iteration 3 only) to
-// dbg_cyc[base + i] and the number of warps to dbg_cyc[base + 4].
-#ifdef PROCLUS_PHASE_PROFILE
-#define PH_DECL()                      \
-  unsigned long long ph_t[4] = {0, 0, 0, 0}; \
-  unsigned long long ph_last = clock64()
-#define PH_MARK(i)                                   \
-  do {                                               \
-    const unsigned long long ph_now = clock64();     \
-    if ((i) >= 0) ph_t[(i) < 0 ? 0 : (i)] += ph_now - ph_last; \
-    ph_last = ph_now;                                \
-  } while (0)
-#define PH_FLUSH(ST, BASE)                                                    \
-  do {                                                                        \
-    if ((threadIdx.x & 31) == 0 && (ST)->iterations == 3) {                   \
-      for (int ph_i = 0; ph_i < 4; ++ph_i) atomicAdd(&(ST)->dbg_cyc[(BASE) + ph_i], ph_t[ph_i]); \
-      atomicAdd(&(ST)->dbg_cyc[(BASE) + 4], 1ull);                            \
-    }                                                                         \
-  } while (0)
-#else
-#define PH_DECL() do {} while (0)
-#define PH_MARK(i) do {} while (0)
-#define PH_FLUSH(ST, BASE) do {} while (0)
-#endif
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -1582,6 +1556,7 @@ __device__ void tail_locality(const RunParams& p, TailMem& T) {
   long long* Hs = (long long*)T.dev;  // [k][d] H rows of MCur by slot
   long long* va = (long long*)T.Z;    // [na][d] band sums by active slot
   state_load(p, S);
+  TST(T, 5);
   const int na = S->n_act;
   for (int c = tid; c < kd; c += bd) {
     const int i = c / d, j = c - i * d;
@@ -1597,6 +1572,7 @@ __device__ void tail_locality(const RunParams& p, TailMem& T) {
     nL_s[tid] = nl;
     cnt_s[tid] = v;
   }
+  TST(T, 8);
   for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
   if (tid == 0 && na > 0)  // byte model: data once + one Dist row per slot
     S->bytes_loc += 4.0 * (double)p.n * (double)(d + (p.variant == 1 ? 0 : na));
@@ -2975,350 +2951,6 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
 #undef LAYK
 }
 
-// --- AssignPoints (Alg 5) + centroid sums (Alg 6 l.1-8), d <= 16: every
-// lane holds the 16 coordinates of 2 point PAIRS in registers (LDS.64 once
-// per pair and dimension) and evaluates seg_{D_c} for all clusters with
-// packed fp32x2 adds (FADD2 with |.|); the medoid rows come from shared
-// memory as warp-broadcast float4s and D_c as a bitmask, so a chunk costs
-// 16 coordinate loads per point instead of one gather per (point, term).
-// Certified fp32 argmin + fp64 fallback (reading R8) as in k_assign; then the
-// chunk is counting-sorted by the new labels and the item threads add the
-// centroid terms.  4 consumer warps x 128 points.
-__global__ void __launch_bounds__(160) k_assign3(RunParams p) {
-#ifdef PROCLUS_PHASE_PROFILE
-  const unsigned long long phs = gtimer();
-#endif
-  DevState* st = p.st;
-  if (st->done) return;
-  extern __shared__ __align__(16) unsigned char smraw[];
-  const SmemLayout& L = p.lay[KK_ASG3];
-  const int P = L.P, d = p.d, k = p.k;
-  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nct = nw * 32;
-  Pipe R = pipe_of(L, smraw, d);
-  __shared__ int off_s[KMAX], nd_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
-  __shared__ float rcp_s[KMAX];
-  __shared__ unsigned msk_s[KMAX];
-  __shared__ int ndmax_s;
-  ItemCtx X = item_ctx(L, smraw, off_s, nd_s, rr_s, ib_s);
-  float* med_s = SMP(float, med);    // [k][16] fp32 rows, zero padded
-  int* dl_s = SMP(int, dl);
-  int* nD_s = SMP(int, nDa);
-  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
-  const long long nmy = chunks_of_block_k(p, P);
-  pipe_init_k(L, R);
-  for (int i = threadIdx.x; i < k; i += blockDim.x) {
-    const int nd = st->nD[i];
-    nD_s[i] = nd;
-    rcp_s[i] = 1.0f / (float)nd;
-    unsigned m = 0;
-    for (int t = 0; t < nd; ++t) m |= 1u << p.dlist[i * d + t];
-    msk_s[i] = m;
-  }
-  for (int e = threadIdx.x; e < k * 16; e += blockDim.x) {
-    const int i = e >> 4, j = e & 15;
-    med_s[e] = j < d ? p.mrows[(long long)st->mcur[i] * d + j] : 0.f;
-  }
-  for (int e = threadIdx.x; e < k * 16; e += blockDim.x) {
-    const int i = e >> 4, t = e & 15;
-    dl_s[e] = t < d ? p.dlist[i * d + t] : 0;  // stride 16, as med_s
-  }
-  items_build<2>(p, L, X);
-  if (threadIdx.x == 0) {
-    int m = 0;
-    for (int i = 0; i < k; ++i) m = max(m, (int)st->nD[i]);
-    ndmax_s = m;
-  }
-  __syncthreads();
-  const double G = (double)(ndmax_s + 6) * 5.9604644775390625e-08;
-  long long nfb = 0;
-#ifdef PROCLUS_PHASE_PROFILE
-  const unsigned long long ph0 = gtimer();
-#endif
-  if (w == nw) {
-    pipe_produce_k(p, R, L, nmy, nullptr);
-  } else {
-    const int tid = w * 32 + lane;
-    const int q0 = w * 128 + 2 * lane;  // pairs (q0, q0+1) and (q0+64, q0+65)
-    long long g0 = (long long)blockIdx.x * P;
-    const long long gstep = (long long)gridDim.x * P;
-    RingPos rp;
-    PH_DECL();
-    for (long long ch = 0; ch < nmy; ++ch, g0 += gstep, rp.next(L.stages)) {
-      PH_MARK(-1);
-      const int stg = rp.stg;
-      const int hb = (int)(ch & 1);
-      int* hist = X.hist0 + hb * KMAX;
-      int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
-      int* list = X.list0 + hb * P;
-      mbar_wait(&R.full[stg], rp.ph);
-      PH_MARK(0);
-      const float* xs = R.buf + (size_t)stg * d * L.ldr;
-      float2 xr[16][2];
-#pragma unroll
-      for (int j = 0; j < 16; ++j)
-#pragma unroll
-        for (int u = 0; u < 2; ++u)
-          xr[j][u] = j < d ? *reinterpret_cast<const float2*>(xs + j * L.ldr + q0 + 64 * u)
-                           : make_float2(0.f, 0.f);
-      float best[4], second[4];
-      int bi[4];
-#pragma unroll
-      for (int v = 0; v < 4; ++v) {
-        best[v] = CUDART_INF_F;
-        second[v] = CUDART_INF_F;
-        bi[v] = 0;
-      }
-      for (int c = 0; c < k; ++c) {
-        const unsigned msk = msk_s[c];
-        const float4* m4 = reinterpret_cast<const float4*>(med_s + c * 16);
-        float2 s0 = make_float2(0.f, 0.f), s1 = s0;
-        // D_c nibble by nibble: one warp-uniform jump per 4 dimensions into a
-        // case that applies exactly the selected dimensions (no predicated
-        // work for the dimensions outside D_c)
-#define NIB_CASE(N, J4)                                                        \
-  case N:                                                                      \
-    if ((N)&1) { s0 = f2_sub_abs_add(s0, xr[4 * J4][0], mv.x); s1 = f2_sub_abs_add(s1, xr[4 * J4][1], mv.x); } \
-    if ((N)&2) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 1][0], mv.y); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 1][1], mv.y); } \
-    if ((N)&4) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 2][0], mv.z); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 2][1], mv.z); } \
-    if ((N)&8) { s0 = f2_sub_abs_add(s0, xr[4 * J4 + 3][0], mv.w); s1 = f2_sub_abs_add(s1, xr[4 * J4 + 3][1], mv.w); } \
-    break;
-#define NIB_SWITCH(J4)                                                         \
-  {                                                                            \
-    const unsigned nib = (msk >> (4 * J4)) & 15u;                              \
-    if (nib) {                                                                 \
-      const float4 mv = m4[J4];                                                \
-      switch (nib) {                                                           \
-        NIB_CASE(1, J4) NIB_CASE(2, J4) NIB_CASE(3, J4) NIB_CASE(4, J4)        \
-        NIB_CASE(5, J4) NIB_CASE(6, J4) NIB_CASE(7, J4) NIB_CASE(8, J4)        \
-        NIB_CASE(9, J4) NIB_CASE(10, J4) NIB_CASE(11, J4) NIB_CASE(12, J4)     \
-        NIB_CASE(13, J4) NIB_CASE(14, J4) NIB_CASE(15, J4)                     \
-        default: break;                                                        \
-      }                                                                        \
-    }                                                                          \
-  }
-        NIB_SWITCH(0) NIB_SWITCH(1) NIB_SWITCH(2) NIB_SWITCH(3)
-#undef NIB_SWITCH
-#undef NIB_CASE
-        const float r = rcp_s[c];
-        const float qv[4] = {s0.x * r, s0.y * r, s1.x * r, s1.y * r};
-#pragma unroll
-        for (int v = 0; v < 4; ++v) {
-          second[v] = qv[v] < best[v] ? best[v] : fminf(second[v], qv[v]);
-          bi[v] = qv[v] < best[v] ? c : bi[v];
-          best[v] = fminf(best[v], qv[v]);
-        }
-      }
-      int qv4[4], cv4[4];
-#pragma unroll
-      for (int v = 0; v < 4; ++v) {
-        const int q = q0 + (v >> 1) * 64 + (v & 1);
-        const long long gp = g0 + q;
-        int lbl = bi[v];
-        if (gp < p.n) {
-          const bool certain = (best[v] >= 1e-30f) && (second[v] < 1e30f) &&
-                               ((double)second[v] * (1.0 - G) > (double)best[v] * (1.0 + G));
-          if (!certain) {
-            lbl = exact_argmin(xs + q, L.ldr, med_s, dl_s, nD_s, k, 16, nullptr, nullptr);
-            ++nfb;
-          }
-        }
-        qv4[v] = q;
-        cv4[v] = gp < p.n ? lbl : -1;
-      }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int q = q0 + 64 * u;
-        const unsigned short two =
-            (unsigned short)((cv4[2 * u] & 0xff) | ((cv4[2 * u + 1] & 0xff) << 8));
-        if (g0 + q + 1 < p.n) {
-          *reinterpret_cast<unsigned short*>(lab + g0 + q) = two;
-        } else if (g0 + q < p.n) {
-          lab[g0 + q] = (unsigned char)cv4[2 * u];
-        }
-      }
-      PH_MARK(1);
-      sort_chunk_m<4>(qv4, cv4, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX, base_s, list);
-      PH_MARK(2);
-      items_chunk<2>(X, reinterpret_cast<const char*>(xs), hist, base_s, list, tid, k);
-      PH_MARK(3);
-      pipe_release(R, stg);
-    }
-    PH_FLUSH(st, 10);
-  }
-#ifdef PROCLUS_PHASE_PROFILE
-  const unsigned long long ph1 = gtimer();
-#endif
-  __syncthreads();
-  items_flush<2>(p, X);
-  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
-#ifdef PROCLUS_PHASE_PROFILE
-  __syncthreads();
-  if (threadIdx.x == 0 && st->iterations == 3) {
-    const unsigned long long ph2 = gtimer();
-    atomicAdd(&st->dbg_cyc[4], ph0 - phs);
-    atomicAdd(&st->dbg_cyc[5], ph1 - ph0);
-    atomicAdd(&st->dbg_cyc[6], ph2 - ph1);
-    atomicAdd(&st->dbg_cyc[7], 1ull);
-    atomicMax(&st->dbg_cyc[8], ~phs);
-    atomicMax(&st->dbg_cyc[9], ph2);
-  }
-#endif
-  if (!p.fuse_tail) return;
-  if (!last_block(&st->ticket[1])) return;
-#define LAYK KK_ASG3
-  RUN_TAIL(tail_assign, 1);
-#undef LAYK
-}
-
-// --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8)
-// on sorted chunks: (1) one thread per point takes the certified fp32
-// argmin of seg_{D_i}(x, m_i) (fp64 fallback near a tie, reading R8) and
-// writes its u8 label; (2) the chunk is counting-sorted by the new labels;
-// (3) the item threads add the centroid terms x_j, j in D_i, exactly.
-__global__ void __launch_bounds__(416) k_assign2(RunParams p) {
-  DevState* st = p.st;
-  if (st->done) return;
-  extern __shared__ __align__(16) unsigned char smraw[];
-  const SmemLayout& L = p.lay[KK_ASG2];
-  const int P = L.P, d = p.d, k = p.k;
-  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int nct = nw * 32;
-  Pipe R = pipe_of(L, smraw, d);
-  __shared__ int off_s[KMAX], nd_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
-  __shared__ float rcp_s[KMAX];
-  __shared__ int ndmax_s;
-  ItemCtx X = item_ctx(L, smraw, off_s, nd_s, rr_s, ib_s);
-  float* med_s = SMP(float, med);
-  Term* tab_s = SMP(Term, tab2);
-  int* dl_s = SMP(int, dl);
-  int* nD_s = SMP(int, nDa);
-  unsigned char* labq = SMP(unsigned char, labq);  // [P] this chunk's labels
-  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
-  const long long nmy = chunks_of_block_k(p, P);
-  pipe_init_k(L, R);
-  for (int i = threadIdx.x; i < k; i += blockDim.x) {
-    const int nd = st->nD[i];
-    nD_s[i] = nd;
-    rcp_s[i] = 1.0f / (float)nd;
-  }
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
-    const int i = e / d;
-    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
-    dl_s[e] = p.dlist[e];
-  }
-  items_build<2>(p, L, X);
-  __syncthreads();
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
-    const int i = e / d, t = e - i * d;
-    if (t < nD_s[i]) {
-      const int j = dl_s[e];
-      tab_s[e].joff = j * L.ldr * 4;
-      tab_s[e].m = med_s[i * d + j];
-    }
-  }
-  if (threadIdx.x == 0) {
-    int m = 0;
-    for (int i = 0; i < k; ++i) m = max(m, nD_s[i]);
-    ndmax_s = m;
-  }
-  __syncthreads();
-  const double G = (double)(ndmax_s + 6) * 5.9604644775390625e-08;
-  long long nfb = 0;
-  if (w == nw) {
-    pipe_produce_k(p, R, L, nmy, nullptr);
-  } else {
-    const int q = w * 32 + lane;
-    long long g0 = (long long)blockIdx.x * P;
-    const long long gstep = (long long)gridDim.x * P;
-    RingPos rp;
-#ifdef PROCLUS_PHASE_PROFILE
-    unsigned long long tw = 0, tdd = 0, tso = 0, tit = 0;
-#endif
-    for (long long ch = 0; ch < nmy; ++ch, g0 += gstep, rp.next(L.stages)) {
-      const int stg = rp.stg;
-      const int hb = (int)(ch & 1);
-      int* hist = X.hist0 + hb * KMAX;
-      int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
-      int* list = X.list0 + hb * P;
-#ifdef PROCLUS_PHASE_PROFILE
-      const unsigned long long c0 = clock64();
-#endif
-      mbar_wait(&R.full[stg], rp.ph);
-#ifdef PROCLUS_PHASE_PROFILE
-      const unsigned long long c1 = clock64();
-      tw += c1 - c0;
-#endif
-      const float* xs = R.buf + (size_t)stg * d * L.ldr;
-      const long long gp = g0 + q;
-      if (gp < p.n) {
-        const float* xq = xs + q;
-        float best = CUDART_INF_F, second = CUDART_INF_F;
-        int bi = 0;
-        const Term* tb = tab_s;
-        for (int c = 0; c < k; ++c, tb += d) {
-          float sv[1];
-          switch (nD_s[c]) {
-#define DT(N) \
-  case N:     \
-    dist_terms<1, N>(xq, tb, sv); \
-    break;
-            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
-            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
-#undef DT
-            default:
-              dist_terms_n<1>(xq, tb, nD_s[c], sv);
-          }
-          const float qv = sv[0] * rcp_s[c];
-          second = qv < best ? best : fminf(second, qv);
-          bi = qv < best ? c : bi;
-          best = fminf(best, qv);
-        }
-        const bool certain = (best >= 1e-30f) && (second < 1e30f) &&
-                             ((double)second * (1.0 - G) > (double)best * (1.0 + G));
-        int lbl = bi;
-        if (!certain) {
-          lbl = exact_argmin(xq, L.ldr, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
-          ++nfb;
-        }
-        lab[gp] = (unsigned char)lbl;
-        labq[q] = (unsigned char)lbl;
-      }
-#ifdef PROCLUS_PHASE_PROFILE
-      const unsigned long long c2 = clock64();
-      tdd += c2 - c1;
-#endif
-      sort_chunk(labq, p.n - g0, q, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX, base_s, list);
-#ifdef PROCLUS_PHASE_PROFILE
-      const unsigned long long c3 = clock64();
-      tso += c3 - c2;
-#endif
-      items_chunk<2>(X, reinterpret_cast<const char*>(xs), hist, base_s, list, q, k);
-#ifdef PROCLUS_PHASE_PROFILE
-      tit += clock64() - c3;
-#endif
-      pipe_release(R, stg);
-    }
-#ifdef PROCLUS_PHASE_PROFILE
-    if (lane == 0 && st->iterations == 3) {
-      atomicAdd(&st->dbg_cyc[10], tw);
-      atomicAdd(&st->dbg_cyc[11], tdd);
-      atomicAdd(&st->dbg_cyc[12], tso);
-      atomicAdd(&st->dbg_cyc[13], tit);
-      atomicAdd(&st->dbg_cyc[14], 1ull);
-    }
-#endif
-  }
-  __syncthreads();
-  items_flush<2>(p, X);
-  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
-  if (!p.fuse_tail) return;
-  if (!last_block(&st->ticket[1])) return;
-#define LAYK KK_ASG2
-  RUN_TAIL(tail_assign, 1);
-#undef LAYK
-}
-
 // --- Final AssignPoints with D* (Alg 1 l.18) and RemoveOutliers (l.19):
 // outlier iff seg_{D*_i}(x, m_i) > Delta_i for every i (reading R17).
 template <int PPT>
@@ -3611,7 +3243,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   // accumulators [nw][cells][32] int64 fit next to the ring
   // sorted-member passes (k_lsum2): 12 consumer warps, chunks of 384 points,
   // ring rows padded by 4 floats (conflict-free row gathers)
-  auto ls2_layout = [&](int ncell, bool asg, int& nw_out) -> SmemLayout {
+  auto ls2_layout = [&](int ncell, int& nw_out) -> SmemLayout {
     SmemLayout best = blank_layout();
     nw_out = 0;
     for (int nw = 12; nw >= 4; nw -= 4) {
@@ -3634,14 +3266,6 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
         L.bal = b.take(4 * 4 * KMAX);
         L.row = b.take(4 * 2 * (size_t)Pk);
         L.cnt = b.take(8 * KMAX);
-        if (asg) {
-          L.lab = -1;
-          L.med = b.take(4 * kd);
-          L.tab2 = b.take(sizeof(Term) * kd);
-          L.dl = b.take(4 * kd);
-          L.nDa = b.take(4 * KMAX);
-          L.labq = b.take((size_t)Pk);
-        }
         finish(L, b, ps.tl);
         if (L.bytes <= 110 * 1024) {
           nw_out = nw;
@@ -3653,46 +3277,14 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   };
   {
     int nw = 0;
-    ps.lay[KK_LS2] = ls2_layout(k * l, false, nw);  // the cost cells: sum |D_i| = k*l
+    ps.lay[KK_LS2] = ls2_layout(k * l, nw);  // the cost cells: sum |D_i| = k*l
     ps.lsum2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
     ps.tpb_ls2 = 32 * (nw + 1);
     ps.smem_ls2 = ps.lsum2 ? ps.lay[KK_LS2].bytes : 0;
-    ps.lay[KK_REF2] = ls2_layout((int)kd, false, nw);
+    ps.lay[KK_REF2] = ls2_layout((int)kd, nw);
     ps.ref2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
     ps.tpb_ref2 = 32 * (nw + 1);
     ps.smem_ref2 = ps.ref2 ? ps.lay[KK_REF2].bytes : 0;
-    {  // k_assign3: 4 consumer warps x 128 points, d <= 16
-      SmemLayout L = blank_layout();
-      LB b;
-      const int nw3 = 4, Pk = 512, stg = 3;
-      const int imax = 32 * nw3 + k * l;
-      L.nw = nw3;
-      L.P = Pk;
-      L.ldr = Pk + 4;
-      L.stages = stg;
-      L.full = b.take(8 * SMAX);
-      L.empty = b.take(8 * SMAX);
-      L.buf = b.take((size_t)stg * d * (Pk + 4) * 4);
-      L.tab = b.take(sizeof(Item) * (size_t)imax);
-      L.acc = b.take(8 * (size_t)imax);
-      L.nD = b.take(4 * kd);
-      L.bal = b.take(4 * 4 * KMAX);
-      L.row = b.take(4 * 2 * (size_t)Pk);
-      L.cnt = b.take(8 * KMAX);
-      L.med = b.take(4 * 16 * (size_t)k);
-      L.dl = b.take(4 * 16 * (size_t)k);
-      L.nDa = b.take(4 * KMAX);
-      L.labq = b.take((size_t)Pk);
-      finish(L, b, ps.tl);
-      ps.lay[KK_ASG3] = L;
-      ps.asg3 = d <= 16 && L.bytes <= 113 * 1024 && getenv("PROCLUS_ASSIGN3");
-      ps.tpb_asg3 = 32 * (nw3 + 1);
-      ps.smem_asg3 = ps.asg3 ? L.bytes : 0;
-    }
-    ps.lay[KK_ASG2] = ls2_layout(k * l, true, nw);
-    ps.asg2 = nw >= 4 && getenv("PROCLUS_ASSIGN2");
-    ps.tpb_asg2 = 32 * (nw + 1);
-    ps.smem_asg2 = ps.asg2 ? ps.lay[KK_ASG2].bytes : 0;
   }
   {  // per-cluster cost pass (k_cost1): lane-private columns [nw][k][32]
     SmemLayout L = blank_layout();
@@ -3751,8 +3343,6 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   ps.grid_fin = grid_of((const void*)k_final<2>, ps.smem_fin, ps.tpb_fin);
   ps.grid_ls2 = ps.lsum2 ? grid_of((const void*)k_lsum2<0>, ps.smem_ls2, ps.tpb_ls2) : 0;
   ps.grid_ref2 = ps.ref2 ? grid_of((const void*)k_lsum2<1>, ps.smem_ref2, ps.tpb_ref2) : 0;
-  ps.grid_asg2 = ps.asg2 ? grid_of((const void*)k_assign2, ps.smem_asg2, ps.tpb_asg2) : 0;
-  ps.grid_asg3 = ps.asg3 ? grid_of((const void*)k_assign3, ps.smem_asg3, ps.tpb_asg3) : 0;
   ps.grid_cost1 = ps.cost1 ? grid_of((const void*)k_cost1, ps.smem_cost1, ps.tpb_cost1) : 0;
   ps.grid = ps.grid_loc;
   ps.per_sm = ps.grid_loc / num_sms;
@@ -3782,19 +3372,9 @@ cudaError_t configure_kernels(const PassShape& ps) {
                              (int)ps.smem_ref2);
     if (e != cudaSuccess) return e;
   }
-  if (ps.asg2) {
-    e = cudaFuncSetAttribute((const void*)k_assign2, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)ps.smem_asg2);
-    if (e != cudaSuccess) return e;
-  }
   if (ps.cost1) {
     e = cudaFuncSetAttribute((const void*)k_cost1, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)ps.smem_cost1);
-    if (e != cudaSuccess) return e;
-  }
-  if (ps.asg3) {
-    e = cudaFuncSetAttribute((const void*)k_assign3, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)ps.smem_asg3);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
@@ -3809,12 +3389,7 @@ void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  if (ps.asg3)
-    k_assign3<<<ps.grid_asg3, ps.tpb_asg3, ps.smem_asg3, s>>>(p);
-  else if (ps.asg2)
-    k_assign2<<<ps.grid_asg2, ps.tpb_asg2, ps.smem_asg2, s>>>(p);
-  else
-    k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
   if (ps.cost1)

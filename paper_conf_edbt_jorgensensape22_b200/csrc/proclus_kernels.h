@@ -19,15 +19,11 @@ struct PassShape {
   size_t smem_loc, smem_asg, smem_cost, smem_ref, smem_fin;
   SmemLayout lay[NLAY];  // per KernelKind
   int lsum2, ref2;       // 1: lane-private accumulator passes (k_lsum2) fit in shared memory
-  int asg2;              // 1: sorted-member assign pass (k_assign2)
-  int asg3;              // 1: register-resident assign pass (k_assign3, d <= 16)
   int cost1;             // 1: per-cluster cost pass (k_cost1)
   int grid_cost1, tpb_cost1;
   size_t smem_cost1;
-  int grid_asg3, tpb_asg3;
-  size_t smem_asg3;
-  int grid_ls2, grid_ref2, grid_asg2, tpb_ls2, tpb_ref2, tpb_asg2;
-  size_t smem_ls2, smem_ref2, smem_asg2;
+  int grid_ls2, grid_ref2, tpb_ls2, tpb_ref2;
+  size_t smem_ls2, smem_ref2;
   TailLayout tl;
   int tail_smem;
 };

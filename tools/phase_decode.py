@@ -1,4 +1,4 @@
-"""Decode the dbg_cyc phase counters printed by tools/phase_prof.sh."""
+"""Decode the dbg_cyc phase counters (tail_cycles line) printed by tools/tail_prof.py."""
 import sys
 
 line = [l for l in open(sys.argv[1]) if l.startswith("tail_cycles")][-1]
