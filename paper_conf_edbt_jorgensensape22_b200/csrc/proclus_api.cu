@@ -564,8 +564,10 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
 // world_size > 1: allreduce the fixed-point cell sums (exact in int64) over
 // NVLink (NCCL), then finalise on every rank.
 static proclus_status split_tail(proclus_handle* h, const RunParams& p, int tail, int iter) {
-  TRY(allreduce(h, p.accg, (size_t)p.k * p.d, ncclInt64));
-  TRY(allreduce(h, p.cntg, KMAX, ncclInt64));
+  // every one of the NCOPY accumulator copies (blocks add into copy
+  // blockIdx % NCOPY; the tail sums the copies), element-wise over ranks
+  TRY(allreduce(h, p.accg, (size_t)NCOPY * p.k * p.d, ncclInt64));
+  TRY(allreduce(h, p.cntg, (size_t)NCOPY * KMAX, ncclInt64));
   launch(h, K_SPLIT, iter, [&] { launch_tail(p, tail, h->stream); });
   return PROCLUS_OK;
 }
@@ -754,7 +756,11 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   p.tl = ps.tl;
   p.tail_smem = ps.tail_smem;
   p.nchunks = (h->n + ps.P - 1) / ps.P;
-  p.fuse_tail = h->world == 1 ? 1 : 0;
+  // PROCLUS_SPLIT_TAIL=1: the multi-GPU schedule (pass, allreduce, separate
+  // tail kernel) on one GPU, so that single-GPU tests cover that path
+  const char* split_env = getenv("PROCLUS_SPLIT_TAIL");
+  const bool force_split = split_env && split_env[0] == '1';
+  p.fuse_tail = (h->world == 1 && !force_split) ? 1 : 0;
   p.cost1 = ps.cost1;
   p.variant = h->variant;
   p.out_labels = h->out_labels.p;
@@ -780,7 +786,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
     const char* v = getenv("PROCLUS_GRAPH");
     return !(v && v[0] == '0');
   }();
-  const bool use_graph = h->world == 1 && !h->stats && graph_env;
+  const bool use_graph = p.fuse_tail && !h->stats && graph_env;
   if (use_graph) {
     // one graph launch: the whole iterative + refinement phase on the device
     TRY(build_graph(h, p, ps));

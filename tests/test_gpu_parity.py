@@ -343,3 +343,27 @@ def test_large_n_properties(pk):
         assert labels[mi] in (i, -1) or sd.shape[0] == 0
     assert (labels >= -1).all() and (labels < k).all()
     assert 6 <= g.iterations < 10000
+
+
+# ------------------------------------------------ multi-GPU schedule on 1 GPU
+# World size > 1 runs every pass without its fused tail, allreduces the
+# fixed-point cell sums (all NCOPY copies) over NCCL and finalises in a
+# separate single-block kernel (split_tail).  PROCLUS_SPLIT_TAIL=1 runs that
+# schedule on one GPU (the allreduce is then the identity), so the tail
+# kernel, the speculative iteration batches and the host control of the
+# N > 1 path are covered by parity here.
+@pytest.mark.parametrize("case", ["C1-1", "C1-2", "C1-3", "C2-1", "shape"])
+def test_split_tail_schedule(pk, orc, monkeypatch, case):
+    monkeypatch.setenv("PROCLUS_SPLIT_TAIL", "1")
+    if case == "shape":
+        data = synth.generate(1500, 100, 5, 33, seed=1500)
+        k, l, seed = 10, 10, 3
+    else:
+        name, seed = case.split("-")
+        seed = int(seed)
+        data, cfg = synth.config_data(name, seed=seed)
+        k, l = cfg["k"], cfg["l"]
+    g, gt, o, ot = run_both(pk, orc, data, k, l, seed=seed)
+    note = assert_parity(g, o, gt, ot, what=f"split tail {case}")
+    if note:
+        pytest.skip(note)
