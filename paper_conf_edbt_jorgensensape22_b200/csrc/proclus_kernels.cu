@@ -771,6 +771,71 @@ static cudaError_t greedy_cluster_np(const double* sT, int nS, int d, int dp, in
   }
 }
 
+// Exact #S x #S sample distances (O0's expression: j ascending, no FMA) by
+// 64 x 64 tiles of the upper triangle, written to both halves (full(p, q)
+// and full(q, p) are bit-identical: the terms are squares / absolute values
+// of negated differences).  A thread keeps 4 x 4 independent accumulation
+// chains, so the 100-step dependent DADD chain of a d = 100 distance is
+// overlapped 16 ways; rows are staged once in shared memory as fp64.
+constexpr int SD_T = 64, SD_J = 32;
+__global__ void __launch_bounds__(256) k_sdist_tiled(const float* __restrict__ srows, int nS,
+                                                     int d, int metric,
+                                                     double* __restrict__ Ds) {
+  __shared__ double sa[SD_J][SD_T], sq[SD_J][SD_T];
+  // upper-triangle tile (ta <= tq) of linear index blockIdx.x
+  const int nt = (nS + SD_T - 1) / SD_T;
+  int t = blockIdx.x, ta = 0;
+  while (t >= nt - ta) {
+    t -= nt - ta;
+    ++ta;
+  }
+  const int tq = ta + t;
+  const int a0 = ta * SD_T, q0 = tq * SD_T;
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  double acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k2 = 0; k2 < 4; ++k2) acc[i][k2] = 0.0;
+  for (int j0 = 0; j0 < d; j0 += SD_J) {
+    __syncthreads();
+    for (int e = threadIdx.x; e < SD_J * SD_T; e += 256) {
+      const int jj = e / SD_T, r = e - jj * SD_T, j = j0 + jj;
+      const int a = a0 + r, q = q0 + r;
+      sa[jj][r] = (j < d && a < nS) ? (double)srows[(long long)a * d + j] : 0.0;
+      sq[jj][r] = (j < d && q < nS) ? (double)srows[(long long)q * d + j] : 0.0;
+    }
+    __syncthreads();
+    const int jn = min(SD_J, d - j0);
+    for (int jj = 0; jj < jn; ++jj) {
+      double va[4], vq[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        va[i] = sa[jj][ty + 16 * i];
+        vq[i] = sq[jj][tx + 16 * i];
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int k2 = 0; k2 < 4; ++k2) {
+          const double u = dsub(vq[k2], va[i]);  // p = S[q], q = S[a] as in O4
+          acc[i][k2] = metric == 1 ? dadd(acc[i][k2], fabs(u)) : dadd(acc[i][k2], dmul(u, u));
+        }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int k2 = 0; k2 < 4; ++k2) {
+      const int a = a0 + ty + 16 * i, q = q0 + tx + 16 * k2;
+      if (a < nS && q < nS) {
+        const double v = metric == 1 ? acc[i][k2] : __dsqrt_rn(acc[i][k2]);
+        Ds[(long long)a * nS + q] = v;
+        Ds[(long long)q * nS + a] = v;
+      }
+    }
+}
+
 cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
                           double* scratch, int* spos, double* pickdist, cudaStream_t s) {
   {  // cluster of 16 CTAs x 64 threads: NP positions per thread
@@ -803,7 +868,12 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
     int blocks = (int)((tot + 255) / 256);
     if (blocks > 148 * 16) blocks = 148 * 16;
     if (blocks < 1) blocks = 1;
-    k_sdist<<<blocks, 256, 0, s>>>(srows, nS, d, metric, scratch);
+    if (getenv("PROCLUS_SDIST_SIMPLE")) {
+      k_sdist<<<blocks, 256, 0, s>>>(srows, nS, d, metric, scratch);
+    } else {
+      const int nt = (nS + SD_T - 1) / SD_T;
+      k_sdist_tiled<<<nt * (nt + 1) / 2, 256, 0, s>>>(srows, nS, d, metric, scratch);
+    }
     k_greedy<<<1, GM_TPB, 0, s>>>(scratch, nS, nM, q0, spos, pickdist);
   } else {
     k_greedy_big<<<1, GR_TPB, sizeof(double) * d, s>>>(srows, nS, d, nM, q0, metric, scratch,
@@ -3144,7 +3214,12 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   }
   ps.P = P;
   ps.stages = stages;
-  const int nw1 = P / 32, nw2 = P / 64;  // consumer warps at 1 / 2 points per lane
+  // consumer warps at 1 point per lane (locality, cost, refinement) and at
+  // PPT2 points per lane (assign, final): 2, or 1 when the chunk is short
+  // (large d) so that a block keeps at least two consumer warps
+  const int ppt2 = P >= 128 ? 2 : 1;
+  const int nw1 = P / 32, nw2 = P / (32 * ppt2);
+  ps.ppt2 = ppt2;
   ps.tpb_loc = 32 * (nw1 + 1);
   ps.tpb_asg = 32 * (nw2 + 1);
   ps.tpb_lsum = 32 * (nw1 + 1);
@@ -3338,9 +3413,11 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
                        : d <= 32 ? (const void*)k_locality<32>
                                  : (const void*)k_locality<0>;
   ps.grid_loc = grid_of(loc_fn, ps.smem_loc, ps.tpb_loc);
-  ps.grid_asg = grid_of((const void*)k_assign<2>, ps.smem_asg, ps.tpb_asg);
+  ps.grid_asg = grid_of(ppt2 == 2 ? (const void*)k_assign<2> : (const void*)k_assign<1>,
+                        ps.smem_asg, ps.tpb_asg);
   ps.grid_lsum = grid_of((const void*)k_labelsum<0>, ps.smem_cost, ps.tpb_lsum);
-  ps.grid_fin = grid_of((const void*)k_final<2>, ps.smem_fin, ps.tpb_fin);
+  ps.grid_fin = grid_of(ppt2 == 2 ? (const void*)k_final<2> : (const void*)k_final<1>,
+                        ps.smem_fin, ps.tpb_fin);
   ps.grid_ls2 = ps.lsum2 ? grid_of((const void*)k_lsum2<0>, ps.smem_ls2, ps.tpb_ls2) : 0;
   ps.grid_ref2 = ps.ref2 ? grid_of((const void*)k_lsum2<1>, ps.smem_ref2, ps.tpb_ref2) : 0;
   ps.grid_cost1 = ps.cost1 ? grid_of((const void*)k_cost1, ps.smem_cost1, ps.tpb_cost1) : 0;
@@ -3355,10 +3432,12 @@ cudaError_t configure_kernels(const PassShape& ps) {
                        (const void*)k_locality<0>,  (const void*)k_assign<2>,
                        (const void*)k_labelsum<0>,  (const void*)k_labelsum<1>,
                        (const void*)k_final<2>,     (const void*)k_prepare,
-                       (const void*)k_tail};
+                       (const void*)k_tail,         (const void*)k_assign<1>,
+                       (const void*)k_final<1>};
   const size_t sm[] = {ps.smem_loc,  ps.smem_loc, ps.smem_loc,   ps.smem_asg, ps.smem_cost,
-                       ps.smem_ref,  ps.smem_fin, (size_t)ps.tail_smem, (size_t)ps.tail_smem};
-  for (int i = 0; i < 9; ++i) {
+                       ps.smem_ref,  ps.smem_fin, (size_t)ps.tail_smem, (size_t)ps.tail_smem,
+                       ps.smem_asg,  ps.smem_fin};
+  for (int i = 0; i < 11; ++i) {
     e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm[i]);
     if (e != cudaSuccess) return e;
   }
@@ -3389,7 +3468,10 @@ void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  if (ps.ppt2 == 2)
+    k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  else
+    k_assign<1><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
   if (ps.cost1)
@@ -3406,7 +3488,10 @@ void launch_refine_x(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_labelsum<1><<<ps.grid_lsum, ps.tpb_lsum, ps.smem_ref, s>>>(p);
 }
 void launch_final(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  k_final<2><<<ps.grid_fin, ps.tpb_fin, ps.smem_fin, s>>>(p);
+  if (ps.ppt2 == 2)
+    k_final<2><<<ps.grid_fin, ps.tpb_fin, ps.smem_fin, s>>>(p);
+  else
+    k_final<1><<<ps.grid_fin, ps.tpb_fin, ps.smem_fin, s>>>(p);
 }
 
 }  // namespace pc

@@ -13,6 +13,7 @@ struct PassShape {
   int P;          // points per chunk
   int stages;     // bulk-copy ring depth
   int tpb_loc, tpb_asg, tpb_lsum, tpb_fin;  // threads per block of each pass
+  int ppt2;       // points per lane of assign / final (2, or 1 for short chunks)
   int per_sm;     // resident blocks per SM (locality)
   int grid;       // persistent blocks (SM count x per_sm)
   int grid_loc, grid_asg, grid_lsum, grid_fin;  // per kernel
