@@ -48,7 +48,7 @@ void launch_gather_m(const float* srows, const long long* sids, const int* spos,
                      float* mrows, long long* mids, cudaStream_t s);
 
 // Small H2D upload through kernel parameters (chunks of BLOB_BYTES).
-constexpr int BLOB_BYTES = 3968;
+constexpr int BLOB_BYTES = 30000;  // < the 32764-byte kernel parameter limit (CUDA >= 12.1)
 void launch_put(void* dst, const void* src, size_t bytes, cudaStream_t s);
 
 PassShape pass_shape(int d, int k, int l, int nM, int num_sms);
