@@ -10,6 +10,17 @@
  *
  * Readings of garbled / silent passages follow SURVEY.md section 8(c) and
  * are listed in DESIGN.md section 3.
+ *
+ * Pins (tests/test_oracle.py, -m "not gpu"): every step below is checked
+ * against something other than itself -- known-answer vectors (SplitMix64),
+ * scipy / numpy (distances, Y / sigma / Z), brute force on tiny inputs
+ * (greedy, delta / L, selection, assignment), the paper's closed forms
+ * (sum Z = 0, sum Z^2 = d - 1; eq 2 = eq 9), worked examples in
+ * tests/golden/, and the FAST-vs-plain equality of Theorems 3.1 / 3.2.
+ * oracle_proclus / oracle_proclus_multi as a whole: parity unpinned by the
+ * paper (it prints no clustering for any input); pinned only through those
+ * steps, the run invariants (disjoint labels, k*l dimensions, >= 2 per
+ * cluster, costBest non-increasing) and the recovery of planted subspaces.
  */
 #ifndef PROCLUS_ORACLE_H
 #define PROCLUS_ORACLE_H
