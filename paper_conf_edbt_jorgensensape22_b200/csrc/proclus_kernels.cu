@@ -3212,6 +3212,9 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     stages = cfg[c][1];
     if ((size_t)stages * (d + k) * P * 4 <= 60 * 1024) break;
   }
+#ifdef PROCLUS_STAGES2
+  if (stages > 2) stages = 2;
+#endif
   ps.P = P;
   ps.stages = stages;
   // consumer warps at 1 point per lane (locality, cost, refinement) and at
