@@ -1052,7 +1052,7 @@ struct Cell {
 // of the warp's points.  fp64 sum (two interleaved accumulators, ascending
 // point order), quantised to int64 at scale 2^e_j and added to the lane's
 // own accumulator.  MODE 0: x, MODE 1: |x - c|.
-template <int MODE, int PPT>
+template <int MODE, int PPT, bool IL = false>
 __device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, int q0,
                                            const Cell* __restrict__ cells, int ncell,
                                            const unsigned* __restrict__ bal,
@@ -1066,16 +1066,17 @@ __device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, 
 #pragma unroll
     for (int u = 0; u < PPT; ++u) {
       unsigned m = bal[C.a * PPT + u];
-      const float* xu = xr + u * 32;
+      // IL: bit b of ballot u is the point 2 b + u (paired points per lane)
+      const float* xu = IL ? xr + u : xr + u * 32;
       while (m) {
         const int b0 = __ffs(m) - 1;
         m &= m - 1u;
-        double v0 = (double)xu[b0];
+        double v0 = (double)xu[IL ? 2 * b0 : b0];
         if (MODE == 1) v0 = fabs(dsub(v0, C.c));
         if (m) {
           const int b1 = __ffs(m) - 1;
           m &= m - 1u;
-          double v1 = (double)xu[b1];
+          double v1 = (double)xu[IL ? 2 * b1 : b1];
           if (MODE == 1) v1 = fabs(dsub(v1, C.c));
           s1 = dadd(s1, v1);
         }
@@ -2244,11 +2245,73 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
 
 // --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8).
 // PPT points per lane so every term-table entry loaded serves PPT points.
-struct __align__(8) Term {
-  int joff;  // byte offset of row j in a ring stage: j * P * 4
-  float m;   // m_ij
+struct __align__(16) Term {
+  float m, m2;  // m_ij twice: one 64-bit operand of the packed subtraction
+  int joff;     // byte offset of row j in a ring stage: j * P * 4
+  int pad;
 };
 #define LDX(base, boff) (*reinterpret_cast<const float*>(reinterpret_cast<const char*>(base) + (boff)))
+
+// Packed fp32 subtraction (FADD2, sm_100): (x0 - m, x1 - m) for a lane's two
+// adjacent points, each half rounded exactly as the scalar fsub_rn.
+__device__ __forceinline__ unsigned long long fsub2(unsigned long long x, unsigned long long m) {
+  unsigned long long r;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(x), "l"(m));
+  return r;
+}
+__device__ __forceinline__ float lo_f(unsigned long long v) { return __uint_as_float((unsigned)v); }
+__device__ __forceinline__ float hi_f(unsigned long long v) {
+  return __uint_as_float((unsigned)(v >> 32));
+}
+#define LDX2(base, boff) \
+  (*reinterpret_cast<const unsigned long long*>(reinterpret_cast<const char*>(base) + (boff)))
+#define TMM(e) (*reinterpret_cast<const unsigned long long*>(&(e).m))
+
+// Paired-point terms (assign, 2 points per lane at xp, xp + 1): one 64-bit
+// shared load and one packed subtraction per term serve both points; the
+// two sums are formed in the same order as dist_terms<2, ND>.
+template <int ND>
+__device__ __forceinline__ void dist_terms2(const float* __restrict__ xp,
+                                            const Term* __restrict__ tb, float (&s)[2]) {
+  float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+#pragma unroll
+  for (int t = 0; t < ND; t += 2) {
+    const Term e0 = tb[t];
+    const unsigned long long r0 = fsub2(LDX2(xp, e0.joff), TMM(e0));
+    a0 += fabsf(lo_f(r0));
+    a1 += fabsf(hi_f(r0));
+    if (t + 1 < ND) {
+      const Term e1 = tb[t + 1];
+      const unsigned long long r1 = fsub2(LDX2(xp, e1.joff), TMM(e1));
+      b0 += fabsf(lo_f(r1));
+      b1 += fabsf(hi_f(r1));
+    }
+  }
+  s[0] = ND > 1 ? a0 + b0 : a0;
+  s[1] = ND > 1 ? a1 + b1 : a1;
+}
+__device__ __noinline__ void dist_terms2_n(const float* __restrict__ xp,
+                                           const Term* __restrict__ tb, int nd, float (&s)[2]) {
+  float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+  int t = 0;
+  for (; t + 2 <= nd; t += 2) {
+    const Term e0 = tb[t], e1 = tb[t + 1];
+    const unsigned long long r0 = fsub2(LDX2(xp, e0.joff), TMM(e0));
+    const unsigned long long r1 = fsub2(LDX2(xp, e1.joff), TMM(e1));
+    a0 += fabsf(lo_f(r0));
+    a1 += fabsf(hi_f(r0));
+    b0 += fabsf(lo_f(r1));
+    b1 += fabsf(hi_f(r1));
+  }
+  if (t < nd) {
+    const Term e = tb[t];
+    const unsigned long long r = fsub2(LDX2(xp, e.joff), TMM(e));
+    a0 += fabsf(lo_f(r));
+    a1 += fabsf(hi_f(r));
+  }
+  s[0] = a0 + b0;
+  s[1] = a1 + b1;
+}
 
 // Segmental distance terms of one cluster for PPT points: fp32 partial sums
 // in two chains (the certified bound only needs the number of terms, DESIGN.md
@@ -2312,7 +2375,6 @@ __device__ __noinline__ void dist_terms_n(const float* __restrict__ xq, const Te
 template <int PPT>
 __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   DevState* st = p.st;
-  if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const SmemLayout& L = p.lay[KK_ASG];
 #define LAYK KK_ASG
@@ -2331,9 +2393,15 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   unsigned* bal_s = SMP(unsigned, bal);
   long long* acc_s = SMP(long long, acc);
   long long* cnt_s = SMP(long long, cnt);
-  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
   const long long nmy = chunks_of_block(p);
-
+  // independent of the previous pass: accumulators, ring, first data copies
+  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
+  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  pipe_init(p, R, nw);
+  __syncthreads();
+  if (st->done) return;
+  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
   for (int i = threadIdx.x; i < k; i += blockDim.x) {
     nD_s[i] = st->nD[i];
     rcp_s[i] = 1.0f / (float)st->nD[i];
@@ -2343,10 +2411,6 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
     dl_s[e] = p.dlist[e];
   }
-  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
-  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
-  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
-  pipe_init(p, R, nw);
   __syncthreads();
   for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
     const int i = e / d, t = e - i * d;
@@ -2354,6 +2418,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
       const int j = dl_s[e];
       tab_s[e].joff = j * P * 4;
       tab_s[e].m = med_s[i * d + j];
+      tab_s[e].m2 = med_s[i * d + j];
     }
   }
   const int ncell = build_cells(cells, nD_s, k, d, off_s, dl_s, nullptr);
@@ -2367,6 +2432,8 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     unsigned* bal = bal_s + w * KMAX * PPT;
     long long* acc = acc_s + (size_t)w * ncap;
     const int q0 = w * 32 * PPT;
+    // PPT == 2: a lane owns the adjacent points q0 + 2 lane + u (packed terms)
+    constexpr bool IL = PPT == 2;
     long long base = (long long)blockIdx.x * P;
     const long long gstep = (long long)gridDim.x * P;
     RingPos rp;
@@ -2374,7 +2441,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
       const int stg = rp.stg;
       mbar_wait(&R.full[stg], rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
-      const float* xq = xs + q0 + lane;
+      const float* xq = xs + q0 + (IL ? 2 * lane : lane);
       float best[PPT], second[PPT];
       int bi[PPT];
 #pragma unroll
@@ -2389,16 +2456,30 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         // fp32 partial sums in any order: the certified bound only needs the
         // number of terms; 4 terms in flight per point
         float s[PPT];
-        switch (nd) {
+        if constexpr (IL) {
+          switch (nd) {
+#define DT(N) \
+  case N:     \
+    dist_terms2<N>(xq, tb, s); \
+    break;
+            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+#undef DT
+            default:
+              dist_terms2_n(xq, tb, nd, s);
+          }
+        } else {
+          switch (nd) {
 #define DT(N) \
   case N:     \
     dist_terms<PPT, N>(xq, tb, s); \
     break;
-          DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
-          DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
 #undef DT
-          default:
-            dist_terms_n<PPT>(xq, tb, nd, s);
+            default:
+              dist_terms_n<PPT>(xq, tb, nd, s);
+          }
         }
         const float r = rcp_s[c];
 #pragma unroll
@@ -2412,7 +2493,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
       int lbl[PPT];
 #pragma unroll
       for (int u = 0; u < PPT; ++u) {
-        const int q = q0 + u * 32 + lane;
+        const int q = IL ? q0 + 2 * lane + u : q0 + u * 32 + lane;
         const long long gp = base + q;
         lbl[u] = -1;
         if (gp >= p.n) continue;
@@ -2446,7 +2527,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         }
       }
       __syncwarp();
-      warp_cells<0, PPT>(xs, P, q0, cells, ncell, bal, acc, scale_s);
+      warp_cells<0, PPT, IL>(xs, P, q0, cells, ncell, bal, acc, scale_s);
       pipe_release(R, stg);
     }
   }
@@ -2947,7 +3028,6 @@ __device__ int cost_qexp(const double* sc, int sgn, const int* dl, const int* nD
 
 __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
   DevState* st = p.st;
-  if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const SmemLayout& L = p.lay[KK_COST1];
 #define LAYK KK_COST1
@@ -2957,11 +3037,13 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
   CItem* tab = SMP(CItem, tab);
   int* nD_s = SMP(int, nD);
   long long* acc_s = SMP(long long, acc);  // [nw][k][32] lane-private columns
-  const unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
   const long long nmy = chunks_of_block(p);
-  for (int i = threadIdx.x; i < k; i += blockDim.x) nD_s[i] = st->nD[i];
   for (int e = threadIdx.x; e < nw * k * 32; e += blockDim.x) acc_s[e] = 0;
   pipe_init(p, R, nw);
+  __syncthreads();
+  if (st->done) return;
+  const unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  for (int i = threadIdx.x; i < k; i += blockDim.x) nD_s[i] = st->nD[i];
   __syncthreads();
   const double sc = scalbn(1.0, cost_qexp(p.scale, 1, p.dlist, nD_s, k, d));
   for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
@@ -3056,6 +3138,7 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
       const int j = dl_s[e];
       tab_s[e].joff = j * P * 4;
       tab_s[e].m = med_s[i * d + j];
+      tab_s[e].m2 = med_s[i * d + j];
     }
   }
   __syncthreads();

@@ -479,7 +479,7 @@ def test_multi_level3_warm_start(orc):
 
 
 def test_multi_level3_grid_shapes(orc):
-    """Level 3 over a grid where k grows and shrinks (top-up from M \ MBest
+    """Level 3 over a grid where k grows and shrinks (top-up from M minus MBest
     and subsets of MBest): invariants of every setting."""
     data = synth.generate(2500, 9, 5, 3, seed=22)
     ks, ls = [3, 5, 2], [2, 4]
