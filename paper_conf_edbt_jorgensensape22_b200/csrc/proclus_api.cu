@@ -129,7 +129,6 @@ struct proclus_handle {
   DBuf<float> srows, mrows;
   DBuf<int> spos;
   DBuf<double> pickdist, gscratch;
-  std::vector<int64_t> h_mids;
   int64_t nS = 0, nM = 0;
   bool m_valid = false;
   uint64_t m_seed = 0;
@@ -148,6 +147,10 @@ struct proclus_handle {
   DBuf<long long> accg, cntg;
   DBuf<DevState> st;
   DevState* h_st = nullptr;  // pinned
+  // pinned staging of the small mid-run / result reads (M ids, D mask): a
+  // pageable D2H would wait behind a prefetch's H2D of the next dataset
+  unsigned char* h_pin = nullptr;
+  size_t h_pin_bytes = 0;
   // graph of one run (prepare -> while{loc, asg, cost} -> refine, final)
   cudaGraphExec_t gexec = nullptr;
   RunParams gkey;
@@ -225,6 +228,18 @@ proclus_status proclus_options_init(proclus_options* opt) {
 }
 
 }  // extern "C"
+
+static proclus_status pin_ensure(proclus_handle* h, size_t bytes) {
+  if (bytes <= h->h_pin_bytes) return PROCLUS_OK;
+  if (h->h_pin) cudaFreeHost(h->h_pin);
+  h->h_pin = nullptr;
+  h->h_pin_bytes = 0;
+  const size_t want = std::max<size_t>(bytes, 4096);
+  if (cudaMallocHost((void**)&h->h_pin, want) != cudaSuccess)
+    return fail(PROCLUS_ENOMEM, "cudaMallocHost(%zu) failed", want);
+  h->h_pin_bytes = want;
+  return PROCLUS_OK;
+}
 
 // N0 pack + per-dimension fixed-point scales.  Cell sums of dimension j are
 // bounded by 2 * n_total * max|x_j| (|x - c| with c inside the column range,
@@ -449,6 +464,7 @@ void proclus_destroy(proclus_handle* h) {
   h->t_bad.release();
   for (cudaEvent_t e : h->evpool) cudaEventDestroy(e);
   if (h->h_st) cudaFreeHost(h->h_st);
+  if (h->h_pin) cudaFreeHost(h->h_pin);
   if (h->comm) ncclCommDestroy(h->comm);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   delete h;
@@ -535,10 +551,8 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
                     h->stream);
   });
   CK(cudaGetLastError());
-  h->h_mids.resize((size_t)nM);
-  CK(cudaMemcpyAsync(h->h_mids.data(), h->mids.p, sizeof(long long) * nM,
-                     cudaMemcpyDeviceToHost, h->stream));
-  CK(cudaStreamSynchronize(h->stream));
+  // no host round trip here: the ids of M are read back with the results
+  // (a mid-run D2H would queue behind a prefetch's H2D on the copy engine)
   h->nS = nS;
   h->nM = nM;
   h->m_valid = true;
@@ -830,17 +844,23 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
     if (out->labels && !out->labels_on_device)
       CK(cudaMemcpyAsync(out->labels, p.out_labels, sizeof(int32_t) * h->n,
                          cudaMemcpyDeviceToHost, h->stream));
+    // pinned staging: [ids of M (int64, #M)][D mask (k x d bytes)]
+    TRY(pin_ensure(h, sizeof(long long) * h->nM + (size_t)k * d));
+    CK(cudaMemcpyAsync(h->h_pin, h->mids.p, sizeof(long long) * h->nM, cudaMemcpyDeviceToHost,
+                       h->stream));
     if (out->dims)
-      CK(cudaMemcpyAsync(out->dims, h->dmask.p, (size_t)k * d, cudaMemcpyDeviceToHost,
-                         h->stream));
+      CK(cudaMemcpyAsync(h->h_pin + sizeof(long long) * h->nM, h->dmask.p, (size_t)k * d,
+                         cudaMemcpyDeviceToHost, h->stream));
   }
   CK(cudaStreamSynchronize(h->stream));
+  if (out && out->dims) memcpy(out->dims, h->h_pin + sizeof(long long) * h->nM, (size_t)k * d);
   if (h->h_st->err) return fail(PROCLUS_EINTERNAL, "device reported error %d", h->h_st->err);
   const int T = h->h_st->iterations;
   if (use_graph) h->launches += 1 + 3 * (int64_t)T + 2;
   if (out) {
     for (int i = 0; i < k; ++i)
-      if (out->medoids) out->medoids[i] = h->h_mids[(size_t)h->h_st->mbest[i]];
+      if (out->medoids)
+        out->medoids[i] = reinterpret_cast<const long long*>(h->h_pin)[h->h_st->mbest[i]];
     out->cost = h->h_st->cost_best;
     out->iterations = T;
   }

@@ -51,3 +51,33 @@ print("load after a finished prefetch ms", round(sum(pl2() for _ in range(10)) /
 x = torch.from_numpy(data).cuda()
 hd = pk.Proclus(x)
 print("device-resident load (pack+scales) ms", round(t(lambda: hd.load(x)), 3))
+
+
+def step_parts(reps=10):
+    """host time of each call of a pipelined step (prefetch, run, load)"""
+    acc = [0.0, 0.0, 0.0]
+    for r in range(reps + 1):
+        t0 = time.perf_counter()
+        h.prefetch(pinned.numpy())
+        t1 = time.perf_counter()
+        h.run(10, 5, seed=3, labels=hlab.numpy())
+        t2 = time.perf_counter()
+        h.load(pinned.numpy())
+        t3 = time.perf_counter()
+        if r:
+            for i, v in enumerate((t1 - t0, t2 - t1, t3 - t2)):
+                acc[i] += v * 1e3 / reps
+    return [round(a, 3) for a in acc]
+
+
+print("step parts (prefetch, run, load) ms", step_parts())
+def run_after_prefetch():
+    h.prefetch(pinned.numpy())
+    t0 = time.perf_counter()
+    h.run(10, 5, seed=3, labels=dlab)
+    t1 = time.perf_counter()
+    h.load(pinned.numpy())
+    return (t1 - t0) * 1e3
+run_after_prefetch()
+print("run (device labels) with a prefetch in flight ms",
+      round(sum(run_after_prefetch() for _ in range(10)) / 10, 3))
