@@ -996,13 +996,14 @@ __device__ bool last_block(unsigned int* ticket) {
 // Combine the per-warp accumulators (exact int64) and add them to one of the
 // NCOPY global copies with one atomic per non-zero cell.  Whole block.
 __device__ void flush_warps(const RunParams& p, const long long* acc_s, int nw, int ncap,
-                            int ncell, const long long* cnt_s, int ncnt) {
+                            int ncell, const long long* cnt_s, int ncnt, int nacc = -1) {
+  if (nacc < 0) nacc = nw;
   const int cp = blockIdx.x % NCOPY;
   long long* acc = p.accg + (size_t)cp * p.k * p.d;
   long long* cnt = p.cntg + (size_t)cp * KMAX;
   for (int c = threadIdx.x; c < ncell; c += blockDim.x) {
     long long s = 0;
-    for (int w = 0; w < nw; ++w) s += acc_s[w * ncap + c];
+    for (int w = 0; w < nacc; ++w) s += acc_s[w * ncap + c];
     if (s) atomicAdd((unsigned long long*)&acc[c], (unsigned long long)s);
   }
   for (int c = threadIdx.x; c < ncnt; c += blockDim.x) {
@@ -1052,7 +1053,7 @@ struct Cell {
 // of the warp's points.  fp64 sum (two interleaved accumulators, ascending
 // point order), quantised to int64 at scale 2^e_j and added to the lane's
 // own accumulator.  MODE 0: x, MODE 1: |x - c|.
-template <int MODE, int PPT, bool IL = false>
+template <int MODE, int PPT, bool IL = false, bool ATOM = false>
 __device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, int q0,
                                            const Cell* __restrict__ cells, int ncell,
                                            const unsigned* __restrict__ bal,
@@ -1084,7 +1085,15 @@ __device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, 
       }
     }
     const double s = dadd(s0, s1);
-    if (s != 0.0) acc[C.acc] += __double2ll_rn(dmul(s, scale_s[C.j]));
+    if (s != 0.0) {
+      const long long v = __double2ll_rn(dmul(s, scale_s[C.j]));
+      // ATOM: one block-wide copy shared by the warps (integer sums: the
+      // order of the additions does not change the total)
+      if (ATOM)
+        atomicAdd((unsigned long long*)&acc[C.acc], (unsigned long long)v);
+      else
+        acc[C.acc] += v;
+    }
   }
 }
 
@@ -2381,6 +2390,10 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   const int P = p.P, d = p.d, k = p.k;
   const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ncap = k * d;
+  // PPT == 1 (long rows, chunk of 2 P): one accumulator copy shared by the
+  // consumer warps (shared-memory atomics) so that 4 of them fit in a block
+  constexpr bool SHACC = PPT == 1;
+  const int nacc = SHACC ? 1 : nw;
   const Pipe R = pipe_of(L, smraw, d);
   float* med_s = SMP(float, med);
   Term* tab_s = SMP(Term, tab);
@@ -2396,7 +2409,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   const long long nmy = chunks_of_block(p);
   // independent of the previous pass: accumulators, ring, first data copies
   for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
-  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nacc * ncap; e += blockDim.x) acc_s[e] = 0;
   for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
   pipe_init(p, R, nw);
   __syncthreads();
@@ -2430,7 +2443,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     pipe_produce(p, R, nmy, nullptr, nullptr);
   } else {
     unsigned* bal = bal_s + w * KMAX * PPT;
-    long long* acc = acc_s + (size_t)w * ncap;
+    long long* acc = acc_s + (SHACC ? (size_t)0 : (size_t)w * ncap);
     const int q0 = w * 32 * PPT;
     // PPT == 2: a lane owns the adjacent points q0 + 2 lane + u (packed terms)
     constexpr bool IL = PPT == 2;
@@ -2527,12 +2540,12 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         }
       }
       __syncwarp();
-      warp_cells<0, PPT, IL>(xs, P, q0, cells, ncell, bal, acc, scale_s);
+      warp_cells<0, PPT, IL, SHACC>(xs, P, q0, cells, ncell, bal, acc, scale_s);
       pipe_release(R, stg);
     }
   }
   __syncthreads();
-  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, k);
+  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, k, nacc);
   if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[1])) return;
@@ -3307,7 +3320,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   const int nw1 = P / 32, nw2 = P / (32 * ppt2);
   ps.ppt2 = ppt2;
   ps.tpb_loc = 32 * (nw1 + 1);
-  ps.tpb_asg = 32 * (nw2 + 1);
+  ps.tpb_asg = 32 * (nw2 + 1);  // updated below when assign takes 2 P
   ps.tpb_lsum = 32 * (nw1 + 1);
   ps.tpb_fin = 32 * (nw2 + 1);
   const size_t kd = (size_t)k * d;
@@ -3337,15 +3350,20 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     finish(L, b, ps.tl);
     ps.lay[KK_LOC] = L;
   }
-  {  // assign
+  // assign: short chunks (ppt2 == 1, long rows) run chunks of 2 P points with
+  // 4 consumer warps sharing one accumulator copy, when that fits (the
+  // per-block cluster tables dominate the shared memory at large k d)
+  auto asg_layout = [&](int Pa) {
+    const int nwa = Pa / (32 * ppt2);
+    const int nacc = ppt2 == 1 ? 1 : nwa;
     SmemLayout L = blank_layout();
     LB b;
-    L.nw = nw2;
-    L.P = P;
-    L.ldr = P;
+    L.nw = nwa;
+    L.P = Pa;
+    L.ldr = Pa;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
-    L.buf = b.take((size_t)stages * d * P * 4);
+    L.buf = b.take((size_t)stages * d * Pa * 4);
     L.med = b.take(4 * kd);
     L.tab = b.take(sizeof(Term) * kd);
     L.dl = b.take(4 * kd);
@@ -3354,11 +3372,20 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.rcp = b.take(4 * KMAX);
     L.scale = b.take(8 * (size_t)d);
     L.cells = b.take(sizeof(Cell) * kd);
-    L.bal = b.take(4 * (size_t)nw2 * KMAX * 2);
-    L.acc = b.take(8 * (size_t)nw2 * kd);
-    L.cnt = b.take(8 * (size_t)nw2 * KMAX);
+    L.bal = b.take(4 * (size_t)nwa * KMAX * 2);
+    L.acc = b.take(8 * (size_t)nacc * kd);
+    L.cnt = b.take(8 * (size_t)nwa * KMAX);
     finish(L, b, ps.tl);
-    ps.lay[KK_ASG] = L;
+    return L;
+  };
+  ps.P_asg = P;
+  ps.lay[KK_ASG] = asg_layout(P);
+  if (ppt2 == 1 && !getenv("PROCLUS_ASG_P1")) {
+    const SmemLayout L2 = asg_layout(2 * P);
+    if (L2.bytes <= 225 * 1024) {  // the 227 KB opt-in limit less static smem
+      ps.P_asg = 2 * P;
+      ps.lay[KK_ASG] = L2;
+    }
   }
   {  // labelsum (cost / refinement X)
     SmemLayout L = blank_layout();
@@ -3468,6 +3495,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   }
   ps.smem_loc = ps.lay[KK_LOC].bytes;
   ps.smem_asg = ps.lay[KK_ASG].bytes;
+  ps.tpb_asg = 32 * (ps.lay[KK_ASG].nw + 1);
   ps.smem_cost = ps.lay[KK_LSUM].bytes;
   ps.smem_ref = ps.smem_cost;
   ps.smem_fin = ps.lay[KK_FIN].bytes;
@@ -3554,10 +3582,16 @@ void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  if (ps.ppt2 == 2)
+  if (ps.ppt2 == 2) {
     k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
-  else
+  } else if (ps.P_asg == p.P) {
     k_assign<1><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
+  } else {  // chunks of P_asg points (same 32-point sub-chunks, same sums)
+    RunParams q = p;
+    q.P = ps.P_asg;
+    q.nchunks = (p.n + q.P - 1) / q.P;
+    k_assign<1><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(q);
+  }
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
   if (ps.cost1)

@@ -14,6 +14,7 @@ struct PassShape {
   int stages;     // bulk-copy ring depth
   int tpb_loc, tpb_asg, tpb_lsum, tpb_fin;  // threads per block of each pass
   int ppt2;       // points per lane of assign / final (2, or 1 for short chunks)
+  int P_asg;      // points per chunk of assign (2 P when ppt2 == 1 and it fits)
   int per_sm;     // resident blocks per SM (locality)
   int grid;       // persistent blocks (SM count x per_sm)
   int grid_loc, grid_asg, grid_lsum, grid_fin;  // per kernel
