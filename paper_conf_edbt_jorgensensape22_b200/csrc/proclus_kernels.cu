@@ -3431,7 +3431,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   // accumulators [nw][cells][32] int64 fit next to the ring
   // sorted-member passes (k_lsum2): 12 consumer warps, chunks of 384 points,
   // ring rows padded by 4 floats (conflict-free row gathers)
-  auto ls2_layout = [&](int ncell, int& nw_out) -> SmemLayout {
+  auto ls2_layout = [&](int ncell, int& nw_out, size_t cap) -> SmemLayout {
     SmemLayout best = blank_layout();
     nw_out = 0;
     for (int nw = 12; nw >= 4; nw -= 4) {
@@ -3455,7 +3455,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
         L.row = b.take(4 * 2 * (size_t)Pk);
         L.cnt = b.take(8 * KMAX);
         finish(L, b, ps.tl);
-        if (L.bytes <= 110 * 1024) {
+        if ((size_t)L.bytes <= cap) {
           nw_out = nw;
           return L;
         }
@@ -3465,11 +3465,14 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   };
   {
     int nw = 0;
-    ps.lay[KK_LS2] = ls2_layout(k * l, nw);  // the cost cells: sum |D_i| = k*l
+    ps.lay[KK_LS2] = ls2_layout(k * l, nw, 110 * 1024);  // the cost cells: sum |D_i| = k*l
     ps.lsum2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
     ps.tpb_ls2 = 32 * (nw + 1);
     ps.smem_ls2 = ps.lsum2 ? ps.lay[KK_LS2].bytes : 0;
-    ps.lay[KK_REF2] = ls2_layout((int)kd, nw);
+    // refinement: two blocks per SM when they fit, else one block with the
+    // largest layout under the opt-in limit (long rows, many cells: C4)
+    ps.lay[KK_REF2] = ls2_layout((int)kd, nw, 110 * 1024);
+    if (nw < 4 && !getenv("PROCLUS_REF_SMALL")) ps.lay[KK_REF2] = ls2_layout((int)kd, nw, 220 * 1024);
     ps.ref2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
     ps.tpb_ref2 = 32 * (nw + 1);
     ps.smem_ref2 = ps.ref2 ? ps.lay[KK_REF2].bytes : 0;
