@@ -836,6 +836,107 @@ __global__ void __launch_bounds__(256) k_sdist_tiled(const float* __restrict__ s
     }
 }
 
+// Greedy over the precomputed exact distance matrix (k_sdist_tiled) with the
+// candidates spread over a cluster of 16 CTAs (NP per thread): every pick
+// each SM reads only its slice of row qs (the single-CTA k_greedy pulls the
+// whole 8 nS-byte row through one SM), and the argmax is exchanged through
+// distributed shared memory exactly as in k_greedy_cluster.  Same keys, same
+// ascending-position tie rule, so the same picks.
+template <int NP>
+__global__ void __launch_bounds__(GC_TPB)
+    k_greedy_mat(const double* __restrict__ Ds, int nS, int nM, int q0, int* __restrict__ spos,
+                 double* __restrict__ pickdist) {
+  constexpr int CS = 16;
+  static_assert(CS * GC_W == 32, "one candidate slot per lane");
+  __shared__ __align__(16) unsigned cand[2][CS * GC_W][4];
+  __shared__ __align__(8) unsigned long long bar[2];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const unsigned rank = cluster_rank();
+  const int g = (int)rank * GC_TPB + tid;
+  if (tid == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  double dreg[NP];
+#pragma unroll
+  for (int t = 0; t < NP; ++t) {
+    const int q = g + t * CS * GC_TPB;
+    dreg[t] = (q < nS && q != q0) ? __ldg(Ds + (long long)q0 * nS + q) : -1.0;
+  }
+  cluster_sync_all();  // every CTA's barriers are initialised before any push
+  if (rank == 0 && tid == 0) {
+    spos[0] = q0;
+    if (pickdist) pickdist[0] = CUDART_INF;
+  }
+  for (int i = 1; i < nM; ++i) {
+    const int par = i & 1;
+    const unsigned ph = (unsigned)(((i - 1) >> 1) & 1);  // use count of slot par
+    if (tid == 0) mbar_expect_tx(&bar[par], CS * GC_W * 16u);
+    unsigned long long bk = 0ull;
+    unsigned bq = 0xffffffffu;
+#pragma unroll
+    for (int t = 0; t < NP; ++t) {
+      const unsigned long long key = dkey(dreg[t]);
+      if (key > bk) {  // ascending position: strict > keeps the smaller one
+        bk = key;
+        bq = g + t * CS * GC_TPB;
+      }
+    }
+    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
+    if (lane < CS)
+      st_async_v4(mapa_u32(smem_u32(&cand[par][rank * GC_W + w][0]), (unsigned)lane), r.hi, r.lo,
+                  r.idx, 0u, mapa_u32(smem_u32(&bar[par]), (unsigned)lane));
+    mbar_wait(&bar[par], ph);
+    KeyIdx sb = warp_argmax(cand[par][lane][0], cand[par][lane][1], cand[par][lane][2]);
+    const int qs = (int)sb.idx;
+    if (rank == 0 && tid == 0) {
+      spos[i] = qs;
+      if (pickdist) {
+        unsigned long long kk = ((unsigned long long)sb.hi << 32) | sb.lo;
+        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
+      }
+    }
+    if (i + 1 < nM) {
+      const double* row = Ds + (long long)qs * nS;
+#pragma unroll
+      for (int t = 0; t < NP; ++t) {
+        const int q = g + t * CS * GC_TPB;
+        if (q == qs) {
+          dreg[t] = -1.0;
+        } else if (dreg[t] >= 0.0) {
+          const double u = __ldg(row + q);
+          if (u < dreg[t]) dreg[t] = u;
+        }
+      }
+    }
+  }
+  cluster_sync_all();  // no CTA leaves while a peer may still push into it
+}
+
+template <int NP>
+static cudaError_t greedy_mat_launch(const double* Ds, int nS, int nM, int q0, int* spos,
+                                     double* pickdist, cudaStream_t s) {
+  constexpr int CS = 16;
+  auto fn = k_greedy_mat<NP>;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(CS, 1, 1);
+  cfg.blockDim = dim3(GC_TPB, 1, 1);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = CS;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, fn, Ds, nS, nM, q0, spos, pickdist);
+}
+
 cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
                           double* scratch, int* spos, double* pickdist, cudaStream_t s) {
   {  // cluster of 16 CTAs x 64 threads: NP positions per thread
@@ -873,6 +974,15 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
     } else {
       const int nt = (nS + SD_T - 1) / SD_T;
       k_sdist_tiled<<<nt * (nt + 1) / 2, 256, 0, s>>>(srows, nS, d, metric, scratch);
+    }
+    const int per = 16 * GC_TPB;
+    const int npm = nS <= 2 * per ? 2 : nS <= 4 * per ? 4 : nS <= 8 * per ? 8 : 0;
+    if (npm && !getenv("PROCLUS_GREEDY_MAT1")) {
+      cudaError_t e = npm == 2   ? greedy_mat_launch<2>(scratch, nS, nM, q0, spos, pickdist, s)
+                      : npm == 4 ? greedy_mat_launch<4>(scratch, nS, nM, q0, spos, pickdist, s)
+                                 : greedy_mat_launch<8>(scratch, nS, nM, q0, spos, pickdist, s);
+      if (e == cudaSuccess) return cudaSuccess;
+      cudaGetLastError();  // cluster launch unavailable: the single-CTA kernel
     }
     k_greedy<<<1, GM_TPB, 0, s>>>(scratch, nS, nM, q0, spos, pickdist);
   } else {
