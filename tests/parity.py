@@ -1,10 +1,15 @@
 """Parity helpers: compare a GPU run with an oracle run on the same seeded
 inputs and RNG streams (north_star contract: labels, medoids and dimension
 sets bit-exact; cost within 1e-5 relative; divergence allowed only at a
-decision the oracle reports as a near tie)."""
+decision the oracle reports as a near tie).
+
+A near-tie divergence never passes silently: ``assert_parity`` calls
+``pytest.skip`` with the iteration, the field and the oracle's margin, so the
+run shows as skipped (not passed) and the reason is in the report."""
 from __future__ import annotations
 
 import numpy as np
+import pytest
 
 NEAR_TIE = 1e-9      # relative Z-selection / cost-comparison gap (SURVEY 8(c) iii)
 COST_RTOL = 1e-5     # north_star tolerance for fp64 sums in a different order
@@ -12,11 +17,15 @@ COST_RTOL = 1e-5     # north_star tolerance for fp64 sums in a different order
 
 def first_divergence(gt, ot):
     """First iteration where the GPU trace and the oracle trace differ, with
-    the oracle's margin there, or None."""
+    the oracle's margin there, or None.  delta_i (Alg 3 l.4-7) is computed
+    in fp64 with the oracle's expression on both sides, so it must be
+    bit-equal."""
     n = min(len(gt.cost), len(ot.cost))
     for it in range(n):
         if not np.array_equal(gt.mcur[it], ot.mcur[it]):
             return it, "mcur", None
+        if not np.array_equal(gt.delta[it], ot.delta[it]):
+            return it, "delta", None
         if not np.array_equal(gt.nL[it], ot.nL[it]):
             return it, "nL", None
         if not np.array_equal(gt.dims[it], ot.dims[it]):
@@ -25,24 +34,28 @@ def first_divergence(gt, ot):
             return it, "sizes", None
         if bool(gt.improved[it]) != bool(ot.improved[it]):
             return it, "improved", float(ot.costgap[it])
+        if not np.array_equal(gt.bad[it], ot.bad[it]):
+            return it, "bad", None
     if len(gt.cost) != len(ot.cost):
         return n, "length", None
     return None
 
 
 def assert_parity(g, o, gt=None, ot=None, what=""):
-    """g/o: results (labels, medoids, dims, cost, iterations); gt/ot traces."""
+    """g/o: results (labels, medoids, dims, cost, iterations); gt/ot traces.
+    Raises on any difference; skips the calling test on an allowed near-tie
+    divergence (oracle margin < NEAR_TIE at the first differing decision)."""
     if gt is not None and ot is not None:
         div = first_divergence(gt, ot)
         if div is not None:
             it, field, margin = div
             if margin is not None and margin < NEAR_TIE:
-                return f"near-tie divergence at iteration {it} ({field}, gap {margin:.3g})"
+                pytest.skip(f"{what}: near-tie divergence at iteration {it} "
+                            f"({field}, oracle gap {margin:.3g} < {NEAR_TIE:g})")
             raise AssertionError(f"{what}: trace diverges at iteration {it} in {field} "
                                  f"(oracle margin {margin})")
         np.testing.assert_allclose(gt.cost, ot.cost, rtol=COST_RTOL, atol=0)
         np.testing.assert_allclose(gt.X, ot.X, rtol=1e-9, atol=1e-12)
-        np.testing.assert_array_equal(gt.bad, ot.bad)
     assert g.iterations == o.iterations, f"{what}: iterations {g.iterations} vs {o.iterations}"
     np.testing.assert_array_equal(g.medoids, o.medoids, err_msg=f"{what}: medoids")
     np.testing.assert_array_equal(g.dims, o.dims, err_msg=f"{what}: dims")
@@ -50,4 +63,3 @@ def assert_parity(g, o, gt=None, ot=None, what=""):
     bad = np.flatnonzero(lab_g != o.labels)
     assert bad.size == 0, f"{what}: {bad.size} labels differ, first at {bad[:5]}"
     np.testing.assert_allclose(g.cost, o.cost, rtol=COST_RTOL, atol=0)
-    return None

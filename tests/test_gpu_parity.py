@@ -34,18 +34,14 @@ def run_both(pk, orc, data, k, l, *, A=100, B=10, minDev=0.7, itrPat=5, seed=1,
 def test_C1_seed_sweep(pk, orc, seed):
     data, cfg = synth.config_data("C1", seed=seed)
     g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
-    note = assert_parity(g, o, gt, ot, what=f"C1 seed {seed}")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"C1 seed {seed}")
 
 
 @pytest.mark.parametrize("seed", range(1, 9))
 def test_C1_L1_metric(pk, orc, seed):
     data, cfg = synth.config_data("C1", seed=seed)
     g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed, metric=1)
-    note = assert_parity(g, o, gt, ot, what=f"C1/L1 seed {seed}")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"C1/L1 seed {seed}")
 
 
 @pytest.mark.parametrize("seed", [1, 2, 3])
@@ -241,15 +237,50 @@ def test_run_multi_levels(pk, orc):
 
 
 # ---------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("metric", [0, 1])
 @pytest.mark.parametrize("name,seed", [("C3", 1), ("C4", 1)])
-def test_full_size_configs(pk, orc, name, seed):
+def test_full_size_configs(pk, orc, name, seed, metric):
     """BASELINE.json full sizes, in the bench's launch configuration: the
-    whole run against the oracle (seconds of CPU each)."""
+    whole run against the oracle (seconds of CPU each), with the paper's
+    Euclidean full-space metric and with north_star's L1
+    (reading R1)."""
     data, cfg = synth.config_data(name, seed=seed)
-    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed)
-    note = assert_parity(g, o, gt, ot, what=name)
-    if note:
-        pytest.skip(note)
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed, metric=metric)
+    assert_parity(g, o, gt, ot, what=f"{name} metric {metric}")
+
+
+# ------------------------------------------------ L1 at every kernel shape
+# The full-space metric enters the greedy (k_greedy_cluster / k_sdist_tiled
+# for DP > 16), the Dist rows of k_locality<16>, <32> and <0> (d <= 16,
+# d <= 32, longer rows) and the exact fp64 fallback.  L1 (north_star) at the
+# d ranges that select each instantiation.
+L1_SHAPES = [
+    # n, d, k, l, A, B
+    (3001, 16, 6, 4, 30, 6),     # k_locality<16>
+    (4097, 33, 8, 6, 20, 5),     # d > 32: k_locality<0>, greedy DP 64
+    (3000, 64, 12, 5, 20, 4),    # d = 64
+    (2600, 100, 10, 10, 20, 5),  # d = 100 (C4 width)
+    (2049, 24, 5, 7, 40, 4),     # d <= 32: k_locality<32>
+]
+
+
+@pytest.mark.parametrize("shape", L1_SHAPES)
+def test_L1_shapes(pk, orc, shape):
+    n, d, k, l, A, B = shape
+    data = synth.generate(n, d, max(2, k // 2), max(2, d // 3), seed=n + d)
+    for seed in (1, 2):
+        g, gt, o, ot = run_both(pk, orc, data, k, l, A=A, B=B, seed=seed, metric=1)
+        assert_parity(g, o, gt, ot, what=f"L1 shape {shape} seed {seed}")
+
+
+@pytest.mark.parametrize("metric", [0, 1])
+def test_greedy_big_sample(pk, orc, metric):
+    """#S > 4096 (k_greedy_big: the sample matrix does not fit the cluster
+    kernels): A*k = 5000 sample points, #M = 250."""
+    data = synth.generate(12000, 6, 8, 3, seed=77)
+    g, gt, o, ot = run_both(pk, orc, data, 25, 3, A=200, B=10, seed=5, metric=metric)
+    assert o.nS == 5000 and o.nM == 250
+    assert_parity(g, o, gt, ot, what=f"greedy big metric {metric}")
 
 
 # ------------------------------------------------ variants (SURVEY 8(f) 1, 2)
@@ -261,9 +292,7 @@ def test_full_size_configs(pk, orc, name, seed):
 def test_variants_C1(pk, orc, variant, seed):
     data, cfg = synth.config_data("C1", seed=seed)
     g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=seed, variant=variant)
-    note = assert_parity(g, o, gt, ot, what=f"variant {variant} C1 seed {seed}")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"variant {variant} C1 seed {seed}")
 
 
 @pytest.mark.parametrize("variant", [1, 2])
@@ -273,9 +302,7 @@ def test_variants_shapes(pk, orc, variant, shape):
     n, d, k, l, A, B = shape
     data = synth.generate(n, d, max(2, k // 2), max(1, d // 3), seed=n)
     g, gt, o, ot = run_both(pk, orc, data, k, l, A=A, B=B, seed=3, variant=variant)
-    note = assert_parity(g, o, gt, ot, what=f"variant {variant} shape {shape}")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"variant {variant} shape {shape}")
 
 
 @pytest.mark.parametrize("variant", [1, 2])
@@ -295,9 +322,7 @@ def test_variants_C2_and_multi(pk, orc, variant):
 def test_variants_full_size_C3(pk, orc, variant):
     data, cfg = synth.config_data("C3", seed=1)
     g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=1, variant=variant)
-    note = assert_parity(g, o, gt, ot, what=f"variant {variant} C3")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"variant {variant} C3")
 
 
 # ------------------------------------------------ n = 8M
@@ -364,6 +389,4 @@ def test_split_tail_schedule(pk, orc, monkeypatch, case):
         data, cfg = synth.config_data(name, seed=seed)
         k, l = cfg["k"], cfg["l"]
     g, gt, o, ot = run_both(pk, orc, data, k, l, seed=seed)
-    note = assert_parity(g, o, gt, ot, what=f"split tail {case}")
-    if note:
-        pytest.skip(note)
+    assert_parity(g, o, gt, ot, what=f"split tail {case}")

@@ -362,8 +362,81 @@ def _check_run_invariants(orc, data, r, k, l, itrPat, n):
         for i in np.flatnonzero(~same):
             assert nxt[i] not in mbest
         assert len(set(nxt.tolist())) == k
-    assert np.array_equal(r.medoids, r.medoids)  # ids returned
     return d
+
+
+def _replay_loop_control(orc, r, n, k, l, minDev, seed):
+    """Replay Alg 1 l.4 and l.10-14 from the trace's cost
+    and cluster sizes alone, with the spec's draws (stream IT, reading R2):
+    the initial MCur (partial Fisher-Yates over [0, #M)), improved = cost <
+    costBest (strict, R14), MBest / sizesBest = MCur / sizes of the last
+    improved iteration, MBad from the sizes of CBest -- the best clustering,
+    Alg 1 l.13 and P:91, reading R11 (not the current iteration's
+    sizes, as Table 1's 'MBad subset of MCur' could be read) -- with
+    thr = n/k*minDev (bad_medoids is pinned by its golden cases), and the
+    replacement of Alg 1 l.14 from M \\ MBest in ascending bad-slot order
+    (R12).  Checks every recorded MCur, improved and MBad against it."""
+    t = r.trace
+    st = orc.stream_it(seed, k, l)
+    pool = list(range(r.nM))
+    for i in range(k):                       # O5: MCur
+        v, st = orc.uniform(st, r.nM - i)
+        j = i + v
+        pool[i], pool[j] = pool[j], pool[i]
+    mcur = np.array(pool[:k])
+    best = np.inf
+    mbest = sizes_best = None
+    for it in range(len(t.cost)):
+        assert np.array_equal(t.mcur[it], mcur), f"MCur at iteration {it}"
+        improved = t.cost[it] < best
+        assert bool(t.improved[it]) == improved, f"improved at iteration {it}"
+        if improved:
+            best = t.cost[it]
+            mbest = mcur.copy()
+            sizes_best = t.sizes[it].copy()
+        bad = orc.bad_medoids(sizes_best, n, minDev)
+        assert np.array_equal(t.bad[it], bad), f"MBad at iteration {it} (from sizesBest)"
+        pool = [q for q in range(r.nM) if q not in set(mbest.tolist())]
+        mcur = mbest.copy()
+        for i in np.flatnonzero(bad):
+            if not pool:
+                break
+            v, st = orc.uniform(st, len(pool))
+            mcur[i] = pool.pop(v)
+    return mbest
+
+
+def _init_M(orc, data, r, k, A, B, seed, metric):
+    """Point ids of M from the pinned pieces (O2-O4): stream SM, the sample
+    S (Alg 1 l.2), the greedy start q0 and Greedy (Alg 2)."""
+    n = data.shape[0]
+    nS = min(A * k, n)
+    st = orc.stream_sm(seed, k)
+    S, st = orc.sample(n, nS, st)
+    q0, st = orc.uniform(st, nS)
+    pos, _ = orc.greedy(data, S, min(B * k, nS), q0, metric)
+    return S[pos]
+
+
+def _check_refinement(orc, data, r, k, l, A, B, seed, metric, mbest):
+    """Alg 1 l.15-19 composed from the pinned pieces: the
+    output medoids are MBest (R16) as point ids; CBest = the assignment of the
+    last improved iteration (its MCur and D); refinement X over CBest
+    with MBest (P:93: 'computing the dimensions using the clusters CBest'),
+    FindDimensions, the final assignment and RemoveOutliers (R17)."""
+    t = r.trace
+    last = int(np.flatnonzero(t.improved)[-1])
+    Mid = _init_M(orc, data, r, k, A, B, seed, metric)
+    assert np.array_equal(r.medoids, Mid[mbest]), "medoids = MBest"
+    med = data[r.medoids]
+    cbest, _ = orc.assign(data, med, t.dims[last])
+    assert np.array_equal(np.bincount(cbest, minlength=k), t.sizes[last])
+    X = orc.cluster_X(data, cbest, med)
+    dstar, _, _ = orc.find_dimensions(X, l)
+    assert np.array_equal(r.dims, dstar), "refined dimensions from CBest / MBest"
+    lab, _ = orc.assign(data, med, dstar)
+    lab, _ = orc.remove_outliers(data, med, dstar, lab)
+    assert np.array_equal(r.labels, lab), "final labels"
 
 
 @pytest.mark.parametrize("seed", range(1, 9))
@@ -371,6 +444,29 @@ def test_run_invariants_C1(orc, seed):
     data, cfg = synth.config_data("C1", seed=seed)
     r = orc.proclus(data, cfg["k"], cfg["l"], seed=seed, trace=True)
     _check_run_invariants(orc, data, r, cfg["k"], cfg["l"], 5, cfg["n"])
+
+
+@pytest.mark.parametrize("metric", [0, 1])
+@pytest.mark.parametrize("seed", range(1, 7))
+def test_loop_control_and_refinement_composed(orc, seed, metric):
+    """The whole run's loop decisions and refinement, recomputed from the
+    pinned pieces (MBad from CBest's sizes, refinement over CBest / MBest).
+    minDev = 1.0 makes MBad non-trivial (several bad slots per iteration)."""
+    data, cfg = synth.config_data("C1", seed=seed)
+    k, l = cfg["k"], cfg["l"]
+    for minDev in (0.7, 1.0):
+        r = orc.proclus(data, k, l, minDev=minDev, seed=seed, metric=metric, trace=True)
+        mbest = _replay_loop_control(orc, r, cfg["n"], k, l, minDev, seed)
+        _check_refinement(orc, data, r, k, l, 100, 10, seed, metric, mbest)
+
+
+def test_loop_control_on_generator_shapes(orc):
+    """Same pins at other shapes (d > 16, k > 8, a small #M pool)."""
+    for (n, d, k, l, A, B, s) in ((3000, 20, 9, 4, 30, 4, 1), (2500, 9, 4, 3, 5, 2, 2)):
+        data = synth.generate(n, d, max(2, k // 2), max(2, d // 4), seed=s)
+        r = orc.proclus(data, k, l, A, B, minDev=0.9, seed=s, trace=True)
+        mbest = _replay_loop_control(orc, r, n, k, l, 0.9, s)
+        _check_refinement(orc, data, r, k, l, A, B, s, 0, mbest)
 
 
 @pytest.mark.parametrize("metric", [0, 1])

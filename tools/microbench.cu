@@ -82,6 +82,47 @@ __global__ void k_lds128(float* out, int stride) {
   out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
 }
 
+__global__ void k_d2ll(long long* out, double a) {
+  double x0 = threadIdx.x * a, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3;
+  long long s0 = 0, s1 = 0, s2 = 0, s3 = 0;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      s0 += __double2ll_rn(x0); s1 += __double2ll_rn(x1);
+      s2 += __double2ll_rn(x2); s3 += __double2ll_rn(x3);
+      x0 += 1.0; x1 += 1.0; x2 += 1.0; x3 += 1.0;
+    }
+  }
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s0 + s1 + s2 + s3;
+}
+
+__global__ void k_f2i(int* out, float a) {
+  float x0 = threadIdx.x * a, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3;
+  int s0 = 0, s1 = 0, s2 = 0, s3 = 0;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      s0 += __float2int_rn(x0); s1 += __float2int_rn(x1);
+      s2 += __float2int_rn(x2); s3 += __float2int_rn(x3);
+      x0 += 1.0f; x1 += 1.0f; x2 += 1.0f; x3 += 1.0f;
+    }
+  }
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s0 + s1 + s2 + s3;
+}
+
+__global__ void k_i64(long long* out, long long a) {
+  long long x0 = threadIdx.x, x1 = x0 + 1, x2 = x0 + 2, x3 = x0 + 3, x4 = x0 + 4, x5 = x0 + 5,
+            x6 = x0 + 6, x7 = x0 + 7;
+  for (int i = 0; i < ITERS; ++i) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      x0 += a; x1 += x0; x2 += a; x3 += x2; x4 += a; x5 += x4; x6 += a; x7 += x6;
+      a ^= x7;
+    }
+  }
+  out[blockIdx.x * blockDim.x + threadIdx.x] = x0 + x1 + x2 + x3 + x4 + x5 + x6 + x7;
+}
+
 int main() {
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
@@ -112,6 +153,9 @@ int main() {
   report("FADD", ITERS * 4.0 * 9, [&] { k_fadd<<<blocks, threads>>>(fo, 1.0f); });
   report("DADD", ITERS * 4.0 * 9, [&] { k_dadd<<<blocks, threads>>>(dout, 1.0); });
   report("F2F+DADD", ITERS * 4.0 * 4, [&] { k_f2f<<<blocks, threads>>>(dout, 1.0f); });
+  report("D2LL", ITERS * 4.0 * 4, [&] { k_d2ll<<<blocks, threads>>>((long long*)dout, 1.0); });
+  report("F2I", ITERS * 4.0 * 4, [&] { k_f2i<<<blocks, threads>>>((int*)fo, 1.0f); });
+  report("I64ADD", ITERS * 4.0 * 9, [&] { k_i64<<<blocks, threads>>>((long long*)dout, 3); });
   report("LDS.32", ITERS * 8.0, [&] { k_lds32<<<blocks, threads>>>(fo, 33); });
   report("LDS.128", ITERS * 8.0, [&] { k_lds128<<<blocks, threads>>>(fo, 9); });
   printf("(LDS rows: loads per thread per s; x4 bytes for .32, x16 for .128)\n");
