@@ -124,6 +124,7 @@ struct proclus_handle {
   DBuf<int> flag;
   DBuf<unsigned> colmax;
   DBuf<double> scale, iscale;
+  int qmagic = 0;  // every 32-point band sum stays below 2^51 at its scale (RunParams::qmagic)
   // init-phase products
   DBuf<long long> sids, mids;
   DBuf<float> srows, mrows;
@@ -272,6 +273,7 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
   CK(cudaStreamSynchronize(h->stream));
   if (bad) return fail(PROCLUS_EINVAL, "data contains non-finite values");
   std::vector<double> sc((size_t)h->d), isc((size_t)h->d);
+  h->qmagic = 1;
   for (int j = 0; j < h->d; ++j) {
     float m;
     memcpy(&m, &cm[(size_t)j], sizeof(float));
@@ -284,6 +286,8 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
       e = std::min(e, 50 - (int)std::ceil(std::log2(2.0 * (double)m)));
       e = std::max(-1000, std::min(1000, e));
     }
+    // a sum of <= 32 terms (<= 64 max|x_j|) below 2^51: quant_sum's fma path
+    if (m > 0.f && std::ldexp(64.0 * (double)m, e) >= std::ldexp(1.0, 51)) h->qmagic = 0;
     sc[(size_t)j] = std::ldexp(1.0, e);
     isc[(size_t)j] = std::ldexp(1.0, -e);
   }
@@ -776,6 +780,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   const bool force_split = split_env && split_env[0] == '1';
   p.fuse_tail = (h->world == 1 && !force_split) ? 1 : 0;
   p.cost1 = ps.cost1;
+  p.qmagic = h->qmagic;
   p.variant = h->variant;
   p.out_labels = h->out_labels.p;
   p.Delta = h->Delta.p;

@@ -117,6 +117,7 @@ struct RunParams {
   long long nchunks;
   int fuse_tail;           // 1: last block finalises (single GPU)
   int cost1;               // 1: the cost pass sums per cluster (k_cost1), cells 0..k-1
+  int qmagic;              // 1: 32-term band sums stay below 2^51 at 2^e_j (quant_sum fma path)
   int variant;             // proclus_variant: 0 FAST, 1 plain (no caches), 2 FAST*
   int use_cond;            // 1: running inside a graph while-node
   unsigned long long cond; // cudaGraphConditionalHandle

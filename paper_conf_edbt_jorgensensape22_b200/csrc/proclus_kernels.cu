@@ -25,6 +25,7 @@
 // graph while-node the cost tail also sets the loop condition.
 #include <math_constants.h>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -50,7 +51,7 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phas
       "{\n"
       ".reg .pred p;\n"
       "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 0x989680;\n"
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(smem_u32(bar)),
       "r"(phase)
@@ -2210,11 +2211,164 @@ __device__ __forceinline__ void band_sums_gen(const float* __restrict__ xs, int 
   }
 }
 
+// Fixed-point quantisation round(s * 2^e_j) of a band / cell sum.  With
+// |s 2^e_j| < 2^51 (p.qmagic, checked on the host for every dimension) one
+// fma with 1.5 * 2^52 rounds to the integer grid exactly as __double2ll_rn
+// (the scale is a power of two, so s * 2^e_j itself is exact), on the fp64
+// pipe instead of the 16/clk/SM conversion pipe.
+__device__ __forceinline__ long long quant_sum(double s, double sc, int magic) {
+  if (magic) {
+    const double v = __fma_rn(s, sc, 6755399441055744.0);  // 1.5 * 2^52
+    return __double_as_longlong(v) - 0x4338000000000000LL;
+  }
+  return __double2ll_rn(dmul(s, sc));
+}
+
+// --- k_locality<16> consumer (d <= 16).  Warp w owns the LOC16_PPT * 32
+// points of columns [w * 32 PPT, (w + 1) * 32 PPT) of every chunk, lane l
+// the points l, l + 32, ...; the active slots are handled one at a time (the
+// loop body is not unrolled over slots: instruction-cache footprint), so the
+// per-slot constants are loaded once per 32 PPT points.  Lane = point for the
+// band decision: the certified fp32 distance (computed for a slot whose Dist
+// row is new, else read from the cached row in the ring), a ballot per point
+// group, and the member's rank, which compacts the members into a per-warp
+// byte list in ascending column order (no bit walks).  Lane = (half h,
+// dimension j) for the band sum of eq 6: half h adds the exact fp64 terms
+// |x_j - m_aj| of the members at ranks h, h + 2, ... (two interleaved
+// accumulators), the halves are added, and the sum is quantised per (slot,
+// dimension, 32 PPT-point group) into the warp's accumulator.  Groups are
+// aligned to 32 PPT points, so the totals do not depend on the grid or on
+// 1024-aligned shard boundaries.
+constexpr int LOC16_PPT = 1;  // 2 measured slower (fewer warps per SM)
+
+// Shared memory is addressed through 32-bit offsets from the dynamic
+// shared-memory base (generic 64-bit pointers cost an IMAD + LEA per access).
+#define SMF(off) (reinterpret_cast<const float*>(smraw)[(off)])
+#define SMB(off) (smraw[(off)])
+
+template <int METRIC>
+__device__ __forceinline__ float loc16_dist(const float (&x)[16], const float* __restrict__ m) {
+  // padded coordinates (j >= d) are 0 in m and in x
+  float s0 = 0.f, s1 = 0.f;
+#pragma unroll
+  for (int j4 = 0; j4 < 4; ++j4) {
+    const float4 v = reinterpret_cast<const float4*>(m)[j4];
+    const float t0 = x[4 * j4] - v.x, t1 = x[4 * j4 + 1] - v.y;
+    const float t2 = x[4 * j4 + 2] - v.z, t3 = x[4 * j4 + 3] - v.w;
+    if (METRIC == 1) {
+      s0 = s0 + fabsf(t0);
+      s1 = s1 + fabsf(t1);
+      s0 = s0 + fabsf(t2);
+      s1 = s1 + fabsf(t3);
+    } else {
+      s0 = __fmaf_rn(t0, t0, s0);
+      s1 = __fmaf_rn(t1, t1, s1);
+      s0 = __fmaf_rn(t2, t2, s0);
+      s1 = __fmaf_rn(t3, t3, s1);
+    }
+  }
+  return METRIC == 1 ? s0 + s1 : sqrtf(s0 + s1);
+}
+
+// buf_f: float offset of the ring; lst_b: byte offset of this warp's list
+template <int METRIC>
+__device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R, int buf_f,
+                                              long long nmy, int na, int ncomp,
+                                              const float* __restrict__ med_s,
+                                              const double* __restrict__ medd_s,
+                                              const int* __restrict__ row_s,
+                                              const Thr* __restrict__ thr_s,
+                                              const ActSlot* __restrict__ act_s, int lst_b,
+                                              long long* __restrict__ acc,
+                                              long long* __restrict__ cnt,
+                                              const double* __restrict__ scale_s, long long& nfb) {
+  extern __shared__ __align__(16) unsigned char smraw[];
+  constexpr int PPT = LOC16_PPT;
+  static_assert(PPT == 1, "x[] holds the coordinates of one point per lane");
+  const int lane = threadIdx.x & 31, c0 = (threadIdx.x >> 5) * 32 * PPT, d = p.d;
+  const int LD = R.ldr, P = p.P, sstride = R.rows * LD;
+  const int h = lane >> 4, j = lane & 15;
+  const unsigned lt = (1u << lane) - 1u;
+  const double sc = scale_s[j < d ? j : 0];
+  const int magic = p.qmagic;
+  const int variant = p.variant;
+  const long long n = p.n, n_pad = p.n_pad;
+  float* const dist = p.dist;
+  long long gp = (long long)blockIdx.x * P + c0 + lane;
+  const long long gstep = (long long)gridDim.x * P;
+  RingPos rp;
+  for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
+    const int stg = rp.stg;
+    mbar_wait(&R.full[stg], rp.ph);
+    const int xs = buf_f + stg * sstride;  // stage base (floats)
+    const int xq = xs + c0 + lane;         // lane's first point, row 0
+    const int xr = xs + j * LD + c0;       // (h, j) view; j >= d: unused rows
+    float x[16];
+    if (ncomp > 0) {  // coordinates in registers when a Dist row is computed; rows >= d are 0
+#pragma unroll
+      for (int jj = 0; jj < 16; ++jj) {
+        const float v = SMF(xq + jj * LD);
+        x[jj] = jj < d ? v : 0.f;
+      }
+    }
+    for (int a = 0; a < na; ++a) {
+      const int rs = row_s[a];
+      const Thr t = thr_s[a];
+      int m = 0;
+#pragma unroll
+      for (int u = 0; u < PPT; ++u) {
+        const bool valid = gp + 32 * u < n;
+        float f;
+        if (rs < 0) {  // a new Dist row
+          f = loc16_dist<METRIC>(x, med_s + a * 16);
+          if (variant != 1 && valid) dist[(long long)act_s[a].key * n_pad + gp + 32 * u] = f;
+        } else {
+          f = SMF(xq + rs + 32 * u);
+        }
+        bool in = f < t.in_hi && f > t.out_lo;
+        if (valid && !in && !(f > t.out_hi || f < t.in_lo)) {
+          // within the fp32 error bound: the oracle's fp64 value decides
+          const ActSlot A = act_s[a];
+          const double dv = full_dist(reinterpret_cast<const float*>(smraw) + xq + 32 * u, LD,
+                                      med_s + a * 16, d, METRIC);
+          in = (dv > A.lo) && (dv <= A.hi);
+          ++nfb;
+        }
+        in = in && valid;
+        const unsigned bl = __ballot_sync(0xffffffffu, in);
+        if (in) smraw[lst_b + m + __popc(bl & lt)] = (unsigned char)(32 * u + lane);
+        m += __popc(bl);
+      }
+      if (m == 0) continue;
+      if (lane == 0) cnt[a] += m;
+      const double c = medd_s[a * 16 + j];
+      __syncwarp();
+      double s0 = 0.0, s1 = 0.0;
+      int v = h;
+#pragma unroll 1
+      for (; v + 2 < m; v += 4) {
+        const double t0 = fabs(dsub((double)SMF(xr + SMB(lst_b + v)), c));
+        const double t1 = fabs(dsub((double)SMF(xr + SMB(lst_b + v + 2)), c));
+        s0 = dadd(s0, t0);
+        s1 = dadd(s1, t1);
+      }
+      if (v < m) s0 = dadd(s0, fabs(dsub((double)SMF(xr + SMB(lst_b + v)), c)));
+      double s = dadd(s0, s1);
+      s = dadd(s, __shfl_xor_sync(0xffffffffu, s, 16));
+      if (h == 0 && j < d && s != 0.0) acc[a * d + j] += quant_sum(s, sc, magic);
+      __syncwarp();  // the list is rewritten by the next slot
+    }
+    pipe_release(R, stg);
+  }
+}
+#undef SMF
+#undef SMB
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
 // One point per lane; the cached Dist rows of the active slots arrive through
 // the same TMA ring as the data (rows d..).  DR: coordinates in registers.
 template <int DR>
-__global__ void __launch_bounds__(288) k_locality(RunParams p) {
+__global__ void __launch_bounds__(288, 3) k_locality(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
@@ -2224,7 +2378,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int na = st->n_act;
   const int ncap = k * d;
-  const Pipe R = pipe_of(L, smraw, d + k);
+  const Pipe R = pipe_of(L, smraw, DR == 16 && d + k < 16 ? 16 : d + k);
   const int LD = R.ldr;
   float* med_s = SMP(float, med);
   ActSlot* act_s = SMP(ActSlot, act);
@@ -2235,6 +2389,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   long long* cnt_s = SMP(long long, cnt);
   ExtraRows* ex = SMP(ExtraRows, ex);
   Thr* thr_s = SMP(Thr, thr);
+  double* medd_s = DR == 16 ? SMP(double, ctr) : nullptr;          // [na][16] fp64 medoid rows
   const long long nmy = chunks_of_block(p);
   const double G = (double)(d + 8) * 5.9604644775390625e-08;  // (d+8) 2^-24
 
@@ -2263,6 +2418,7 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
     const int a = e / MS, j = e - a * MS;
     const float m = j < d ? p.mrows[(long long)act_s[a].mpos * d + j] : 0.f;
     med_s[e] = m;
+    if (DR == 16) medd_s[e] = (double)m;
   }
   __syncthreads();
   long long nfb = 0;
@@ -2271,6 +2427,15 @@ __global__ void __launch_bounds__(288) k_locality(RunParams p) {
   if (na > 0) {
     if (w == nw) {
       pipe_produce(p, R, nmy, nullptr, ex);
+    } else if constexpr (DR == 16) {
+      if (p.metric == 1)
+        loc16_consume<1>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s,
+                         L.tab + w * 32 * LOC16_PPT, acc_s + (size_t)w * ncap, cnt_s + w * KMAX, scale_s,
+                         nfb);
+      else
+        loc16_consume<0>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s,
+                         L.tab + w * 32 * LOC16_PPT, acc_s + (size_t)w * ncap, cnt_s + w * KMAX, scale_s,
+                         nfb);
     } else {
       unsigned* bal = bal_s + w * KMAX;
       long long* acc = acc_s + (size_t)w * ncap;
@@ -3429,7 +3594,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   const int ppt2 = P >= 128 ? 2 : 1;
   const int nw1 = P / 32, nw2 = P / (32 * ppt2);
   ps.ppt2 = ppt2;
-  ps.tpb_loc = 32 * (nw1 + 1);
+  ps.tpb_loc = 32 * ((d <= 16 ? nw1 / LOC16_PPT : nw1) + 1);
   ps.tpb_asg = 32 * (nw2 + 1);  // updated below when assign takes 2 P
   ps.tpb_lsum = 32 * (nw1 + 1);
   ps.tpb_fin = 32 * (nw2 + 1);
@@ -3439,7 +3604,8 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   {  // locality
     SmemLayout L = blank_layout();
     LB b;
-    L.nw = nw1;
+    // d <= 16: LOC16_PPT points per lane (k_locality<16>), fewer consumer warps
+    L.nw = d <= 16 ? nw1 / LOC16_PPT : nw1;
     L.P = P;
     // rows padded by 4 floats so that the lane-per-dimension band sums of
     // k_locality read a point's coordinates with at most 2- (d <= 16) or
@@ -3447,7 +3613,8 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.ldr = P + 4;
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
-    L.buf = b.take((size_t)stages * (d + k) * L.ldr * 4);
+    // >= 16 rows: k_locality<16> loads rows 0..15 of every stage unconditionally
+    L.buf = b.take((size_t)stages * std::max(d + k, 16) * L.ldr * 4);
     L.med = b.take(4 * (size_t)k * (d < 32 ? 32 : d));  // rows padded to 16 / 32
     L.act = b.take(sizeof(ActSlot) * KMAX);
     L.row = b.take(4 * KMAX);
@@ -3457,6 +3624,10 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.cnt = b.take(8 * (size_t)nw1 * KMAX);
     L.ex = b.take(sizeof(ExtraRows));
     L.thr = b.take(sizeof(Thr) * KMAX);
+    if (d <= 16) {
+      L.ctr = b.take(8 * (size_t)k * 16);        // fp64 medoid rows of the d <= 16 consumer
+      L.tab = b.take((size_t)nw1 * 32);          // per-warp member lists (32 PPT points)
+    }
     finish(L, b, ps.tl);
     ps.lay[KK_LOC] = L;
   }
