@@ -46,6 +46,7 @@ extern "C" {
 #define PROCLUS_D_MAX 256  /* a 2-stage ring of 64-point chunks fits in SMEM */
 
 typedef struct proclus_handle proclus_handle;
+typedef struct proclus_group proclus_group;
 
 typedef enum {
   PROCLUS_OK = 0,
@@ -83,6 +84,9 @@ typedef struct {
   int32_t variant;         /* proclus_variant: which caches the iterative
                               phase keeps; every variant returns the same
                               clustering                     */
+  proclus_group* group;    /* world_size > 1 without NCCL: the in-process
+                              communicator from proclus_group_create (then
+                              nccl_unique_id is ignored); NULL: NCCL        */
 } proclus_options;
 
 /* GPU-FAST-PROCLUS (default): the Dist row of every potential medoid is
@@ -147,6 +151,21 @@ typedef struct {
   int64_t fallbacks[4];   /* exact fp64 re-decisions (locality, assign,
                              final): points within the fp32 error bound    */
 } proclus_stats;
+
+/* In-process communicator for `world` row shards whose handles live in ONE
+ * process (any devices, also several shards on one GPU: test layer F of
+ * SURVEY 4.2).  Pass it as options.group with options.world_size = world and
+ * a distinct options.rank per handle.  Each rank's proclus_create_ex /
+ * proclus_run / proclus_run_multi must then be called from its own host
+ * thread, the ranks with identical arguments except data and labels: the
+ * calls rendezvous at every collective.  The partial sums (int64 fixed-point
+ * cells, counts, per-dimension maxima, gathered sample rows) are combined
+ * by a host-staged reduction in rank order, so the results are bit-identical
+ * to the NCCL path and to world_size 1.
+ * EINVAL: world < 1 or > 1024, out == NULL.  The caller destroys the group
+ * after every handle that uses it (proclus_group_destroy is NULL-safe). */
+PROCLUS_API proclus_status proclus_group_create(int32_t world, proclus_group** out);
+PROCLUS_API void proclus_group_destroy(proclus_group* g);
 
 /* Fill *opt with defaults (device -1, L2, max_iter 10000, host data, own
  * stream, no trace, world_size 1). */

@@ -40,7 +40,7 @@ class proclus_options(C.Structure):
                 ("data_on_device", C.c_int32), ("stream", C.c_void_p), ("trace", C.c_int32),
                 ("world_size", C.c_int32), ("rank", C.c_int32), ("n_global", C.c_int64),
                 ("row_offset", C.c_int64), ("nccl_unique_id", C.c_void_p),
-                ("stats", C.c_int32), ("variant", C.c_int32)]
+                ("stats", C.c_int32), ("variant", C.c_int32), ("group", C.c_void_p)]
 
 
 STAT_KINDS = ["pack", "gather", "greedy", "prepare", "locality", "assign", "cost",
@@ -70,6 +70,8 @@ class proclus_trace(C.Structure):
 # every entry point of include/proclus.h: (name, restype, argtypes)
 SIGNATURES = [
     ("proclus_options_init", C.c_int, [C.POINTER(proclus_options)]),
+    ("proclus_group_create", C.c_int, [C.c_int32, C.POINTER(C.c_void_p)]),
+    ("proclus_group_destroy", None, [C.c_void_p]),
     ("proclus_create", C.c_int, [C.c_void_p, C.c_int64, C.c_int32, C.POINTER(C.c_void_p)]),
     ("proclus_create_ex", C.c_int, [C.c_void_p, C.c_int64, C.c_int32,
                                     C.POINTER(proclus_options), C.POINTER(C.c_void_p)]),
@@ -117,6 +119,16 @@ def proclus_options_init() -> proclus_options:
     o = proclus_options()
     _check(lib().proclus_options_init(C.byref(o)))
     return o
+
+
+def proclus_group_create(world: int) -> C.c_void_p:
+    g = C.c_void_p()
+    _check(lib().proclus_group_create(world, C.byref(g)))
+    return g
+
+
+def proclus_group_destroy(g):
+    lib().proclus_group_destroy(g)
 
 
 def _ptr(a) -> int:
@@ -217,7 +229,8 @@ class Proclus:
                  max_iter: int = 0, trace: bool = False, stream: int | None = None,
                  stats: bool = False, variant: int = VARIANT_FAST,
                  world_size: int = 1, rank: int = 0, n_global: int = 0,
-                 row_offset: int = 0, nccl_unique_id: bytes | None = None):
+                 row_offset: int = 0, nccl_unique_id: bytes | None = None,
+                 group=None):
         on_dev = hasattr(data, "is_cuda") and bool(data.is_cuda)
         if on_dev:
             if data.dtype.__str__() != "torch.float32" or not data.is_contiguous():
@@ -245,9 +258,13 @@ class Proclus:
         if nccl_unique_id is not None:
             self._uid = C.create_string_buffer(bytes(nccl_unique_id), 128)
             o.nccl_unique_id = C.cast(self._uid, C.c_void_p)
+        if group is not None:
+            o.group = group.value if isinstance(group, C.c_void_p) else group
         self.options = o
+        self._on_dev = on_dev
         self.h = proclus_create_ex(data, self.n, self.d, o)
         self._k = None
+        self._pf = None  # the array of a pending prefetch (kept alive)
 
     def close(self):
         if getattr(self, "h", None):
@@ -266,18 +283,65 @@ class Proclus:
     def __exit__(self, *exc):
         self.close()
 
+    def _device_index(self) -> int:
+        return int(self.options.device) if self.options.device >= 0 else _current_device()
+
+    def _checked_data(self, data, copy_ok: bool):
+        """The C ABI reads n*d floats from the pointer (host or device per
+        the handle): shape, dtype, contiguity and residency are checked here."""
+        if self._on_dev:
+            if not (hasattr(data, "is_cuda") and data.is_cuda):
+                raise ValueError("this handle was created with device data: pass a CUDA tensor")
+            if str(data.dtype) != "torch.float32" or not data.is_contiguous():
+                raise ValueError("device data must be a contiguous float32 tensor")
+            if data.device.index != self._device_index():
+                raise ValueError(f"tensor on cuda:{data.device.index}, handle on "
+                                 f"cuda:{self._device_index()}")
+            if tuple(data.shape) != (self.n, self.d):
+                raise ValueError(f"data shape {tuple(data.shape)} != ({self.n}, {self.d})")
+            return data
+        if hasattr(data, "is_cuda") and data.is_cuda:
+            raise ValueError("this handle was created with host data: pass a host array")
+        if hasattr(data, "numpy"):
+            data = data.numpy()
+        arr = np.asarray(data)
+        if not copy_ok and (arr.dtype != np.float32 or not arr.flags.c_contiguous):
+            raise ValueError("prefetch needs a C-contiguous float32 array (no copy is made)")
+        arr = np.ascontiguousarray(arr, dtype=np.float32)
+        if arr.shape != (self.n, self.d):
+            raise ValueError(f"data shape {arr.shape} != ({self.n}, {self.d})")
+        return arr
+
     def load(self, data):
-        if not hasattr(data, "data_ptr"):
-            data = np.ascontiguousarray(data, dtype=np.float32)
+        data = self._checked_data(data, copy_ok=True)
         proclus_load(self.h, data)
+        self._pf = None  # the prefetched buffer is no longer referenced by the library
 
     def prefetch(self, data):
-        """Start the H2D copy of the next dataset (keep `data` alive and
-        unchanged until load(data) returns); load(data) then waits for it."""
+        """Start the H2D copy of the next dataset (keep `data` unchanged until
+        load(data) returns); load(data) then waits for it.  The handle keeps a
+        reference to `data` until then."""
+        if self._on_dev:
+            raise ValueError("prefetch is for handles with host data")
+        data = self._checked_data(data, copy_ok=False)
         proclus_prefetch(self.h, data)
+        self._pf = data
 
     def _result_struct(self, k, labels=None):
         on_dev = labels is not None and hasattr(labels, "is_cuda") and bool(labels.is_cuda)
+        if labels is not None:
+            if on_dev:
+                if str(labels.dtype) != "torch.int32" or not labels.is_contiguous():
+                    raise ValueError("device labels must be a contiguous int32 tensor")
+                if labels.device.index != self._device_index():
+                    raise ValueError("labels tensor on another device than the handle")
+                if labels.numel() < self.n:
+                    raise ValueError(f"labels holds {labels.numel()} < n = {self.n} elements")
+            else:
+                if (not isinstance(labels, np.ndarray) or labels.dtype != np.int32
+                        or not labels.flags.c_contiguous or labels.size < self.n):
+                    raise ValueError("host labels must be a C-contiguous int32 ndarray of "
+                                     f">= n = {self.n} elements")
         if labels is None:
             labels = np.empty(self.n, np.int32)
         med = np.empty(k, np.int64)
@@ -337,6 +401,12 @@ class Proclus:
     @property
     def last_launches(self) -> int:
         return proclus_last_launches(self.h)
+
+
+def _current_device() -> int:
+    import torch
+
+    return int(torch.cuda.current_device())
 
 
 def proclus(data, k: int, l: int, A: int = 100, B: int = 10, minDev: float = 0.7,

@@ -7,6 +7,10 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <condition_variable>
+#include <mutex>
+#include <new>
+
 #include <algorithm>
 #include <cmath>
 #include <cstdarg>
@@ -102,6 +106,31 @@ enum Kind {
   K_PACK = 0, K_GATHER, K_GREEDY, K_PREPARE, K_LOC, K_ASG, K_COST, K_REF, K_FIN, K_SPLIT
 };
 
+// In-process communicator of `world` handles (test layer F): the
+// shards' partial sums are combined by a host-staged reduction in fixed rank
+// order, so the row-sharded schedule runs with G logical shards on one GPU
+// and no NCCL.  Every rank calls the collectives from its own host thread;
+// they rendezvous at a generation-counted barrier.
+struct proclus_group {
+  int world = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  long long gen = 0;
+  std::vector<std::vector<unsigned char>> slot;  // per rank: this collective's bytes
+  void barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    const long long g = gen;
+    if (++arrived == world) {
+      arrived = 0;
+      ++gen;
+      cv.notify_all();
+    } else {
+      cv.wait(lk, [&] { return gen != g; });
+    }
+  }
+};
+
 struct proclus_handle {
   int dev = 0;
   cudaStream_t stream = nullptr;
@@ -113,6 +142,7 @@ struct proclus_handle {
   int variant = 0;  // proclus_variant
   int world = 1, rank = 0;
   ncclComm_t comm = nullptr;
+  proclus_group* group = nullptr;  // in-process communicator (instead of comm)
   int num_sms = 148;
   int64_t launches = 0;
 
@@ -205,10 +235,48 @@ static proclus_status set_device(proclus_handle* h) {
   return PROCLUS_OK;
 }
 
+// Element-wise reduction of the ranks' slots in rank order 0, 1, ... (sum or
+// max; the int64 cell sums are exact, the float sum adds one non-zero row).
+template <class T>
+static void group_reduce(proclus_group* g, size_t count, bool is_max, T* out) {
+  for (size_t e = 0; e < count; ++e) {
+    T acc = reinterpret_cast<const T*>(g->slot[0].data())[e];
+    for (int r = 1; r < g->world; ++r) {
+      const T v = reinterpret_cast<const T*>(g->slot[(size_t)r].data())[e];
+      acc = is_max ? (v > acc ? v : acc) : (T)(acc + v);
+    }
+    out[e] = acc;
+  }
+}
+
 static proclus_status allreduce(proclus_handle* h, void* buf, size_t count, ncclDataType_t t,
                                 ncclRedOp_t op = ncclSum) {
   if (h->world <= 1) return PROCLUS_OK;
-  CKN(ncclAllReduce(buf, buf, count, t, op, h->comm, h->stream));
+  if (!h->group) {
+    CKN(ncclAllReduce(buf, buf, count, t, op, h->comm, h->stream));
+    return PROCLUS_OK;
+  }
+  size_t es = 0;
+  switch (t) {
+    case ncclInt64: es = 8; break;
+    case ncclUint32: case ncclInt32: case ncclFloat: es = 4; break;
+    default: return fail(PROCLUS_EINTERNAL, "group allreduce: unsupported type");
+  }
+  proclus_group* g = h->group;
+  std::vector<unsigned char> res(count * es);
+  g->slot[(size_t)h->rank].resize(count * es);
+  CK(cudaMemcpyAsync(g->slot[(size_t)h->rank].data(), buf, count * es, cudaMemcpyDeviceToHost,
+                     h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  g->barrier();  // every rank's slot is filled
+  const bool mx = op == ncclMax;
+  if (t == ncclInt64) group_reduce(g, count, mx, reinterpret_cast<long long*>(res.data()));
+  else if (t == ncclUint32) group_reduce(g, count, mx, reinterpret_cast<unsigned*>(res.data()));
+  else if (t == ncclInt32) group_reduce(g, count, mx, reinterpret_cast<int*>(res.data()));
+  else group_reduce(g, count, mx, reinterpret_cast<float*>(res.data()));
+  g->barrier();  // every rank has read every slot
+  CK(cudaMemcpyAsync(buf, res.data(), count * es, cudaMemcpyHostToDevice, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
   return PROCLUS_OK;
 }
 
@@ -217,6 +285,20 @@ extern "C" {
 const char* proclus_last_error(void) { return g_err.c_str(); }
 int32_t proclus_abi_version(void) { return PROCLUS_ABI_VERSION; }
 int32_t proclus_target_sm(void) { return 100; }
+
+proclus_status proclus_group_create(int32_t world, proclus_group** out) {
+  if (!out) return fail(PROCLUS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (world < 1 || world > 1024) return fail(PROCLUS_EINVAL, "world must be in [1, 1024]");
+  proclus_group* g = new (std::nothrow) proclus_group;
+  if (!g) return fail(PROCLUS_ENOMEM, "group allocation");
+  g->world = world;
+  g->slot.resize((size_t)world);
+  *out = g;
+  return PROCLUS_OK;
+}
+
+void proclus_group_destroy(proclus_group* g) { delete g; }
 
 proclus_status proclus_options_init(proclus_options* opt) {
   if (!opt) return fail(PROCLUS_EINVAL, "opt is NULL");
@@ -364,7 +446,12 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
       return cleanup(fail(PROCLUS_ECUDA, "cudaStreamCreate failed"));
     h->own_stream = true;
   }
-  if (h->world > 1) {
+  if (h->world > 1 && o.group) {
+    proclus_group* g = reinterpret_cast<proclus_group*>(o.group);
+    if (g->world != h->world)
+      return cleanup(fail(PROCLUS_EINVAL, "group of %d ranks, world_size %d", g->world, h->world));
+    h->group = g;
+  } else if (h->world > 1) {
     if (!o.nccl_unique_id) return cleanup(fail(PROCLUS_EINVAL, "nccl_unique_id required"));
     ncclUniqueId id;
     memcpy(&id, o.nccl_unique_id, sizeof(id));
