@@ -226,6 +226,23 @@ PROCLUS_API proclus_status proclus_run_multi(proclus_handle* h, const int32_t* k
                                  int32_t itrPat, uint64_t seed,
                                  int32_t reuse_level, proclus_result* outs);
 
+/* A list of independent settings (ks[s], ls[s]), s < nset, for
+ * splitting a multi-parameter grid across GPUs or processes (settings
+ * parallelism: every rank holds the whole dataset, no communication).
+ * reuse_level 1: every setting equals proclus_run(ks[s], ls[s], seed).
+ * reuse_level 2: S and M are drawn once for k_sample (>= every ks[s]) and
+ *   the caches are shared, so outs[s] equals the result of that setting in
+ *   proclus_run_multi(..., reuse_level 2) over any grid whose largest k is
+ *   k_sample -- whichever rank runs it.
+ * Level 3 (warm starts from the previous setting) is sequential and not
+ * offered here.
+ * EINVAL: nset < 1, reuse_level not in {1,2}, an invalid (k, l), k_sample
+ * smaller than some ks[s] or outside [2, PROCLUS_K_MAX] (level 2). */
+PROCLUS_API proclus_status proclus_run_list(proclus_handle* h, const int32_t* ks,
+                                const int32_t* ls, int32_t nset, int32_t k_sample,
+                                int32_t A, int32_t B, double minDev, int32_t itrPat,
+                                uint64_t seed, int32_t reuse_level, proclus_result* outs);
+
 /* Copy the trace of the last run (requires options.trace = 1). */
 PROCLUS_API proclus_status proclus_get_trace(proclus_handle* h, proclus_trace* tr);
 

@@ -82,6 +82,9 @@ SIGNATURES = [
     ("proclus_run_multi", C.c_int, [C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p, C.c_int32,
                                     C.c_int32, C.c_int32, C.c_double, C.c_int32, C.c_uint64,
                                     C.c_int32, C.POINTER(proclus_result)]),
+    ("proclus_run_list", C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_int32,
+                                   C.c_int32, C.c_int32, C.c_double, C.c_int32, C.c_uint64,
+                                   C.c_int32, C.POINTER(proclus_result)]),
     ("proclus_get_trace", C.c_int, [C.c_void_p, C.POINTER(proclus_trace)]),
     ("proclus_get_stats", C.c_int, [C.c_void_p, C.POINTER(proclus_stats)]),
     ("proclus_last_launches", C.c_int64, [C.c_void_p]),
@@ -167,6 +170,15 @@ def proclus_run_multi(h, ks, ls, A, B, minDev, itrPat, seed, reuse_level, outs):
     ls = np.ascontiguousarray(ls, np.int32)
     _check(lib().proclus_run_multi(h, ks.ctypes.data, len(ks), ls.ctypes.data, len(ls),
                                    A, B, minDev, itrPat, seed, reuse_level, outs))
+
+
+def proclus_run_list(h, ks, ls, k_sample, A, B, minDev, itrPat, seed, reuse_level, outs):
+    ks = np.ascontiguousarray(ks, np.int32)
+    ls = np.ascontiguousarray(ls, np.int32)
+    if ks.shape != ls.shape:
+        raise ValueError("ks and ls must have the same length")
+    _check(lib().proclus_run_list(h, ks.ctypes.data, ls.ctypes.data, len(ks), k_sample, A, B,
+                                  minDev, itrPat, seed, reuse_level, outs))
 
 
 def proclus_get_trace(h, tr: proclus_trace):
@@ -366,6 +378,23 @@ class Proclus:
                 outs[a * len(ls) + b] = r
                 keep.append((lab, med, dims))
         proclus_run_multi(self.h, ks, ls, A, B, minDev, itrPat, seed, reuse_level, outs)
+        return [Result(lab, med, dims.astype(bool), float(outs[i].cost), int(outs[i].iterations))
+                for i, (lab, med, dims) in enumerate(keep)]
+
+    def run_list(self, settings, k_sample: int, A=100, B=10, minDev=0.7, itrPat=5, seed=1,
+                 reuse_level: int = 2) -> list[Result]:
+        """Independent settings [(k, l), ...] (settings parallelism): level 2
+        draws S and M once for k_sample, so each result equals that
+        setting of run_multi over a grid with largest k = k_sample."""
+        settings = [(int(k), int(l)) for k, l in settings]
+        outs = (proclus_result * len(settings))()
+        keep = []
+        for i, (k, _) in enumerate(settings):
+            r, lab, med, dims = self._result_struct(k)
+            outs[i] = r
+            keep.append((lab, med, dims))
+        proclus_run_list(self.h, [k for k, _ in settings], [l for _, l in settings], k_sample,
+                         A, B, minDev, itrPat, seed, reuse_level, outs)
         return [Result(lab, med, dims.astype(bool), float(outs[i].cost), int(outs[i].iterations))
                 for i, (lab, med, dims) in enumerate(keep)]
 

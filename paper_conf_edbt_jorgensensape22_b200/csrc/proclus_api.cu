@@ -888,10 +888,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   // graph mode unless per-launch events are wanted, multi-GPU (NCCL between
   // kernels), or PROCLUS_GRAPH=0 (ncu cannot profile kernels of graphs that
   // contain conditional nodes)
-  static const bool graph_env = [] {
-    const char* v = getenv("PROCLUS_GRAPH");
-    return !(v && v[0] == '0');
-  }();
+  const char* genv = getenv("PROCLUS_GRAPH");
+  const bool graph_env = !(genv && genv[0] == '0');
   const bool use_graph = p.fuse_tail && !h->stats && graph_env;
   if (use_graph) {
     // one graph launch: the whole iterative + refinement phase on the device
@@ -1037,6 +1035,33 @@ proclus_status proclus_run_multi(proclus_handle* h, const int32_t* ks, int32_t n
                       reuse_level == 3 ? &warm : nullptr));
       if (reuse_level == 3) warm.assign(h->h_st->mbest, h->h_st->mbest + ks[a]);
     }
+  return PROCLUS_OK;
+}
+
+proclus_status proclus_run_list(proclus_handle* h, const int32_t* ks, const int32_t* ls,
+                                int32_t nset, int32_t k_sample, int32_t A, int32_t B,
+                                double minDev, int32_t itrPat, uint64_t seed,
+                                int32_t reuse_level, proclus_result* outs) {
+  if (!h || !ks || !ls || !outs) return fail(PROCLUS_EINVAL, "NULL argument");
+  if (nset < 1) return fail(PROCLUS_EINVAL, "empty settings list");
+  if (reuse_level != 1 && reuse_level != 2)
+    return fail(PROCLUS_EINVAL, "reuse_level must be 1 or 2 (level 3 is sequential)");
+  for (int s = 0; s < nset; ++s) {
+    TRY(validate_setting(h, ks[s], ls[s], A, B, minDev, itrPat));
+    if (reuse_level == 2 && ks[s] > k_sample)
+      return fail(PROCLUS_EINVAL, "k_sample %d < k = %d of setting %d", k_sample, ks[s], s);
+    if (!outs[s].labels || !outs[s].medoids || !outs[s].dims)
+      return fail(PROCLUS_EINVAL, "outs[%d] arrays are required", s);
+  }
+  if (reuse_level == 2 && (k_sample < 2 || k_sample > PROCLUS_K_MAX))
+    return fail(PROCLUS_EINVAL, "k_sample must be in [2, %d]", PROCLUS_K_MAX);
+  TRY(set_device(h));
+  reset_stats(h);
+  if (reuse_level == 2) TRY(init_phase(h, k_sample, A, B, seed));
+  for (int s = 0; s < nset; ++s) {
+    if (reuse_level == 1) TRY(init_phase(h, ks[s], A, B, seed));
+    TRY(run_setting(h, ks[s], ls[s], minDev, itrPat, seed, &outs[s]));
+  }
   return PROCLUS_OK;
 }
 

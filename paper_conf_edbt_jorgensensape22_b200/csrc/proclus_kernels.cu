@@ -1578,6 +1578,7 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
         }
         const unsigned before = x - tot;
         const int need = need_s;
+        __syncwarp();  // every lane has read need_s before one lane rewrites it
         const bool here = (int)before < need && need <= (int)x;
         const unsigned who = __ballot_sync(0xffffffffu, here);
         if (here && tid == __ffs(who) - 1) {
@@ -1980,6 +1981,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
     // replacement draws (stream IT): the r-th remaining pool entry, in order;
     // every lane runs the same generator, the removal shift is warp-wide
     unsigned long long rng = S->rng;
+    __syncwarp();  // every lane has read S->rng before lane 0 stores it back
     for (int i = 0; i < k; ++i) {
       if (!((bad >> i) & 1u) || np == 0) continue;
       const int r = (int)sm64_uniform(&rng, (unsigned long long)np);

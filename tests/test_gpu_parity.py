@@ -390,3 +390,52 @@ def test_split_tail_schedule(pk, orc, monkeypatch, case):
         k, l = cfg["k"], cfg["l"]
     g, gt, o, ot = run_both(pk, orc, data, k, l, seed=seed)
     assert_parity(g, o, gt, ot, what=f"split tail {case}")
+
+
+# ------------------------------------------------ settings parallelism (C5)
+@pytest.mark.parametrize("level", [1, 2])
+def test_run_list_splits_grid(pk, orc, level):
+    """The C5 sweep split across ranks: every rank holds the whole
+    dataset and runs its share of the (k, l) settings through run_list with
+    k_sample = the grid's largest k; the union equals run_multi over the grid
+    bit for bit, and the oracle's multi-parameter run."""
+    data = synth.generate(6000, 10, 5, 3, seed=12)
+    ks, ls = [3, 4, 5], [2, 3, 4]
+    with pk.Proclus(data) as h:
+        whole = h.run_multi(ks, ls, seed=7, reuse_level=level)
+    settings = [(k, l) for k in ks for l in ls]
+    got = [None] * len(settings)
+    for rank in range(3):  # three "ranks", one after the other on this GPU
+        mine = list(range(rank, len(settings), 3))
+        with pk.Proclus(data) as h:
+            res = h.run_list([settings[i] for i in mine], k_sample=max(ks), seed=7,
+                             reuse_level=level)
+        for i, r in zip(mine, res):
+            got[i] = r
+    want = orc.proclus_multi(data, ks, ls, seed=7, reuse_level=level)
+    for i, (g, w, o) in enumerate(zip(got, whole, want)):
+        assert np.array_equal(g.labels, w.labels) and np.array_equal(g.medoids, w.medoids)
+        assert np.array_equal(g.dims, w.dims) and g.cost == w.cost
+        assert g.iterations == w.iterations
+        assert_parity(g, o, what=f"run_list level {level} setting {settings[i]}")
+
+
+# ------------------------------------------------ SURVEY 8(f) row 4: oracle parity at n = 8M
+@pytest.mark.parametrize("k,l", [(10, 5), (15, 7)])
+def test_L8_oracle_parity(pk, orc, k, l):
+    """Fig 3e's large-n workload (> 8M points) against the oracle: the
+    default setting (L8) and one setting of the 9-setting grid (L8S, reading
+    R22), full traces, labels, medoids, dimensions, iterations and cost.  The
+    plain oracle needs ~2 minutes of one host core per run."""
+    import torch
+
+    data, cfg = synth.config_data("L8", seed=1)
+    x = torch.from_numpy(data).cuda()
+    lab = torch.empty(data.shape[0], dtype=torch.int32, device="cuda")
+    with pk.Proclus(x, trace=True) as h:
+        g = h.run(k, l, seed=1, labels=lab)
+        gt = h.trace()
+    g.labels = lab.cpu().numpy()
+    del x
+    o = orc.proclus(data, k, l, seed=1, trace=True)
+    assert_parity(g, o, gt, o.trace, what=f"L8 k={k} l={l}")
