@@ -719,12 +719,16 @@ static proclus_status build_graph(proclus_handle* h, RunParams p, const PassShap
   cudaGraph_t body = cp.conditional.phGraph_out[0];
   CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
   launch_locality(p, ps, cs);
+  if (!p.fuse_tail) launch_tail(p, TAIL_LOC, cs);
   launch_assign(p, ps, cs);
+  if (!p.fuse_tail) launch_tail(p, TAIL_ASG, cs);
   launch_cost(p, ps, cs);
+  if (!p.fuse_tail) launch_tail(p, TAIL_COST, cs);
   CK(cudaStreamEndCapture(cs, &tmp));
   // refinement after the loop
   CK(cudaStreamBeginCaptureToGraph(cs, g, &wnode, nullptr, 1, cudaStreamCaptureModeRelaxed));
   launch_refine_x(p, ps, cs);
+  if (!p.fuse_tail) launch_tail(p, TAIL_REF, cs);
   launch_final(p, ps, cs);
   CK(cudaStreamEndCapture(cs, &tmp));
   CK(cudaStreamDestroy(cs));
@@ -865,7 +869,12 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   // tail kernel) on one GPU, so that single-GPU tests cover that path
   const char* split_env = getenv("PROCLUS_SPLIT_TAIL");
   const bool force_split = split_env && split_env[0] == '1';
-  p.fuse_tail = (h->world == 1 && !force_split) ? 1 : 0;
+  // PROCLUS_TAIL_KERNELS=1: single GPU with the single-block tails as kernels
+  // of their own (the north_star's separate Z-score / selection kernel)
+  // instead of the last block of each pass; graph mode still applies
+  const char* tk_env = getenv("PROCLUS_TAIL_KERNELS");
+  const bool tail_kernels = h->world == 1 && tk_env && tk_env[0] == '1';
+  p.fuse_tail = (h->world == 1 && !force_split && !tail_kernels) ? 1 : 0;
   p.cost1 = ps.cost1;
   p.qmagic = h->qmagic;
   p.variant = h->variant;
@@ -890,7 +899,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   // contain conditional nodes)
   const char* genv = getenv("PROCLUS_GRAPH");
   const bool graph_env = !(genv && genv[0] == '0');
-  const bool use_graph = p.fuse_tail && !h->stats && graph_env;
+  const bool use_graph = (p.fuse_tail || tail_kernels) && !h->stats && graph_env;
   if (use_graph) {
     // one graph launch: the whole iterative + refinement phase on the device
     TRY(build_graph(h, p, ps));
@@ -946,7 +955,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   if (out && out->dims) memcpy(out->dims, h->h_pin + sizeof(long long) * h->nM, (size_t)k * d);
   if (h->h_st->err) return fail(PROCLUS_EINTERNAL, "device reported error %d", h->h_st->err);
   const int T = h->h_st->iterations;
-  if (use_graph) h->launches += 1 + 3 * (int64_t)T + 2;
+  if (use_graph) h->launches += p.fuse_tail ? 1 + 3 * (int64_t)T + 2 : 1 + 6 * (int64_t)T + 3;
   if (out) {
     for (int i = 0; i < k; ++i)
       if (out->medoids)

@@ -57,6 +57,31 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phas
       "r"(phase)
       : "memory");
 }
+// the same with the barrier's 32-bit shared address computed once per kernel
+// (a generic-to-shared conversion per spin iteration costs an S2UR chain)
+__device__ __forceinline__ void mbar_wait(unsigned bar, unsigned phase) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAITA_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 0x989680;\n"
+      "@!p bra WAITA_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(phase)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes,
+                                         unsigned bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(bar)
+      : "memory");
+}
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes,
                                          unsigned long long* bar) {
   asm volatile(
@@ -1002,6 +1027,9 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
 __device__ __forceinline__ void mbar_arrive(unsigned long long* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
 
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
@@ -1026,6 +1054,7 @@ struct Pipe {
   unsigned long long* empty;  // [SMAX]
   int rows;
   int ldr;                    // row stride in floats (>= P)
+  unsigned full_a, empty_a;   // 32-bit shared addresses of full[0] / empty[0]
 };
 
 __device__ __forceinline__ void pipe_init(const RunParams& p, const Pipe& R, int nw) {
@@ -1048,19 +1077,19 @@ __device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
   int stg = 0, round = 0;
   for (long long i = 0; i < nmy; ++i) {
     if (round > 0) {  // the consumers of chunk i - stages released this stage
-      mbar_wait(&R.empty[stg], (unsigned)((round - 1) & 1));
+      mbar_wait(R.empty_a + 8u * stg, (unsigned)((round - 1) & 1));
       fence_proxy_async();
     }
     const long long base = (blockIdx.x + i * gridDim.x) * (long long)p.P;
-    if (lane == 0) mbar_expect_tx(&R.full[stg], bytes);
+    if (lane == 0) mbar_expect_tx(R.full_a + 8u * stg, bytes);
     __syncwarp();
     float* dst = R.buf + (size_t)stg * R.rows * R.ldr;
     for (int j = lane; j < p.d + nex; j += 32) {
       const float* src = j < p.d ? p.xs + (size_t)j * p.n_pad + base : ex->src[j - p.d] + base;
-      bulk_g2s(dst + (size_t)j * R.ldr, src, row, &R.full[stg]);
+      bulk_g2s(dst + (size_t)j * R.ldr, src, row, R.full_a + 8u * stg);
     }
     if (labsrc && lane == 0)
-      bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, &R.full[stg]);
+      bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, R.full_a + 8u * stg);
     if (++stg == p.stages) {
       stg = 0;
       ++round;
@@ -1083,7 +1112,7 @@ struct RingPos {
 
 __device__ __forceinline__ void pipe_release(const Pipe& R, int stg) {
   __syncwarp();
-  if ((threadIdx.x & 31) == 0) mbar_arrive(&R.empty[stg]);
+  if ((threadIdx.x & 31) == 0) mbar_arrive(R.empty_a + 8u * stg);
 }
 
 // The last block to arrive (ticket) returns true; it then sees every other
@@ -1244,6 +1273,8 @@ __device__ Pipe carve_pipe(Carve& cv, const RunParams& p, int rows, bool with_la
   R.empty = cv.take<unsigned long long>(SMAX);
   R.buf = cv.take<float>((size_t)p.stages * rows * p.P);
   R.lab = with_lab ? cv.take<unsigned char>((size_t)p.stages * p.P) : nullptr;
+  R.full_a = smem_u32(R.full);
+  R.empty_a = smem_u32(R.empty);
   return R;
 }
 
@@ -1512,36 +1543,70 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
   }
   __syncthreads();
   TST(T, tq < 0 ? 3 : tq);
-  for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
-    const int j1 = warp_argmin_row(key + i * d, d, -1);
-    const int j2 = warp_argmin_row(key + i * d, d, j1);
-    if (lane == 0) {
-      dm[i * d + j1] = 1;
-      dm[i * d + j2] = 1;
+  const int R = k * l - 2 * k;
+  if (d <= 64) {
+    // two smallest per row by (key, j), one thread per row: a sequential
+    // scan of d shared keys beats two warp reductions per row here
+    if (tid < k) {
+      const unsigned long long* kr = key + tid * d;
+      unsigned long long b1 = ~0ull, b2 = ~0ull;
+      int j1 = 0, j2 = 1;
+      for (int j = 0; j < d; ++j) {  // ascending j: strict < keeps the smaller j on ties
+        const unsigned long long v = kr[j];
+        if (v < b1) {
+          b2 = b1;
+          j2 = j1;
+          b1 = v;
+          j1 = j;
+        } else if (v < b2) {
+          b2 = v;
+          j2 = j;
+        }
+      }
+      dm[tid * d + j1] = 1;
+      dm[tid * d + j2] = 1;
+      if (R > 0) {  // taken cells never rank before a free one
+        key[tid * d + j1] = ~0ull;
+        key[tid * d + j2] = ~0ull;
+      }
     }
+  } else {
+    for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
+      const int j1 = warp_argmin_row(key + i * d, d, -1);
+      const int j2 = warp_argmin_row(key + i * d, d, j1);
+      if (lane == 0) {
+        dm[i * d + j1] = 1;
+        dm[i * d + j2] = 1;
+      }
+    }
+    __syncthreads();
+    if (R > 0 && kd <= 512)
+      for (int c = tid; c < kd; c += bd)
+        if (dm[c]) key[c] = ~0ull;  // taken: never before a free cell
   }
   __syncthreads();
   TST(T, tq < 0 ? 4 : tq);
-  const int R = k * l - 2 * k;
-  if (R > 0 && kd <= 512) {  // rank by a scan over all keys: O(kd^2 / threads)
-    for (int c = tid; c < kd; c += bd)
-      if (dm[c]) key[c] = ~0ull;  // taken: never before a free cell
-    __syncthreads();
+  if (R > 0 && kd <= 512) {
+    // rank of every free cell among the free cells by (key, i, j) = (key,
+    // cell index): O(kd^2 / threads) broadcast reads, two keys per load
+    const ulonglong2* key2 = reinterpret_cast<const ulonglong2*>(key);
+    const int kd2 = kd >> 1;
     for (int c = tid; c < kd; c += bd) {
-      if (dm[c]) continue;
       const unsigned long long kc = key[c];
-      int rank = 0;
-      int o = 0;
-      for (; o + 4 <= kd; o += 4) {
-        const unsigned long long k0 = key[o], k1 = key[o + 1], k2 = key[o + 2], k3 = key[o + 3];
-        rank += (k0 < kc || (k0 == kc && o < c)) + (k1 < kc || (k1 == kc && o + 1 < c)) +
-                (k2 < kc || (k2 == kc && o + 2 < c)) + (k3 < kc || (k3 == kc && o + 3 < c));
+      if (kc == ~0ull) continue;
+      int r0 = 0, r1 = 0;
+#pragma unroll 4
+      for (int o2 = 0; o2 < kd2; ++o2) {
+        const ulonglong2 v = key2[o2];
+        const int o = 2 * o2;
+        r0 += (v.x < kc) | ((v.x == kc) & (o < c));
+        r1 += (v.y < kc) | ((v.y == kc) & (o + 1 < c));
       }
-      for (; o < kd; ++o) {
-        const unsigned long long ko = key[o];
-        rank += (ko < kc || (ko == kc && o < c));
+      if (kd & 1) {
+        const unsigned long long v = key[kd - 1];
+        r0 += (v < kc) | ((v == kc) & (kd - 1 < c));
       }
-      if (rank < R) dm[c] = 1;
+      if (r0 + r1 < R) dm[c] = 1;
     }
   } else if (R > 0) {
     __shared__ unsigned int hist[256];
@@ -1965,34 +2030,55 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
     if (lane < k) S->mcur[lane] = S->mbest[lane];
     __syncwarp();
     TSTW(T, 13);
-    // pool = ascending positions of M not in MBest
-    int np = 0;
-    for (int t0 = 0; t0 < nM; t0 += 32) {
-      const int t = t0 + lane;
-      bool inb = t >= nM;
-      if (!inb)
-        for (int i = 0; i < k; ++i) inb |= (S->mbest[i] == t);
-      const unsigned b = __ballot_sync(full, !inb);
-      if (!inb) T.pool[np + __popc(b & ((1u << lane) - 1u))] = t;
-      np += __popc(b);
+    // pool = ascending positions of M not in MBest, as a bitmap in shared
+    // memory (word w holds positions 32 w .. 32 w + 31); the r-th remaining
+    // pool entry is found by a warp prefix count of the words' populations
+    // and a find-n-th-set-bit, and removed by clearing its bit -- the same
+    // draws as erasing it from the ascending list (reading R12)
+    unsigned* avail = reinterpret_cast<unsigned*>(T.pool);
+    const int nwrd = (nM + 31) >> 5;
+    for (int w0 = lane; w0 < nwrd; w0 += 32) {
+      const int rem = nM - 32 * w0;
+      avail[w0] = rem >= 32 ? 0xffffffffu : ((1u << rem) - 1u);
     }
     __syncwarp();
+    if (lane < k) atomicAnd(&avail[S->mbest[lane] >> 5], ~(1u << (S->mbest[lane] & 31)));
+    __syncwarp();
+    int np = nM - k;  // MBest holds k distinct positions of M
     TSTW(T, 18);
     // replacement draws (stream IT): the r-th remaining pool entry, in order;
-    // every lane runs the same generator, the removal shift is warp-wide
+    // every lane runs the same generator
     unsigned long long rng = S->rng;
     __syncwarp();  // every lane has read S->rng before lane 0 stores it back
     for (int i = 0; i < k; ++i) {
       if (!((bad >> i) & 1u) || np == 0) continue;
-      const int r = (int)sm64_uniform(&rng, (unsigned long long)np);
-      if (lane == 0) S->mcur[i] = T.pool[r];
-      for (int t0 = r; t0 < np - 1; t0 += 32) {
-        const int t = t0 + lane;
-        const int v = t < np - 1 ? T.pool[t + 1] : 0;
-        __syncwarp();
-        if (t < np - 1) T.pool[t] = v;
-        __syncwarp();
+      int r = (int)sm64_uniform(&rng, (unsigned long long)np);
+      int pos = -1;
+      for (int w0 = 0; w0 < nwrd && pos < 0; w0 += 32) {
+        const unsigned wv = w0 + lane < nwrd ? avail[w0 + lane] : 0u;
+        const int c = __popc(wv);
+        int x = c;  // inclusive prefix count over the lanes of this group
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(full, x, o);
+          if (lane >= o) x += y;
+        }
+        const unsigned hit = __ballot_sync(full, r < x && r >= x - c);
+        if (hit) {
+          const int src = __ffs(hit) - 1;
+          const int before = __shfl_sync(full, x - c, src);
+          const unsigned sw = __shfl_sync(full, wv, src);
+          const int bit = __fns(sw, 0, r - before + 1);
+          pos = 32 * (w0 + src) + bit;
+        } else {
+          r -= __shfl_sync(full, x, 31);
+        }
       }
+      if (lane == 0) {
+        S->mcur[i] = pos;
+        avail[pos >> 5] &= ~(1u << (pos & 31));
+      }
+      __syncwarp();
       --np;
     }
     TSTW(T, 19);
@@ -2083,6 +2169,8 @@ __device__ __forceinline__ Pipe pipe_of(const SmemLayout& L, unsigned char* smra
   R.lab = L.lab >= 0 ? SMP(unsigned char, lab) : nullptr;
   R.rows = rows;
   R.ldr = L.ldr > 0 ? L.ldr : L.P;
+  R.full_a = smem_u32(R.full);
+  R.empty_a = smem_u32(R.empty);
   return R;
 }
 
@@ -2245,8 +2333,20 @@ constexpr int LOC16_PPT = 1;  // 2 measured slower (fewer warps per SM)
 
 // Shared memory is addressed through 32-bit offsets from the dynamic
 // shared-memory base (generic 64-bit pointers cost an IMAD + LEA per access).
-#define SMF(off) (reinterpret_cast<const float*>(smraw)[(off)])
-#define SMB(off) (smraw[(off)])
+// explicit 32-bit shared-window addressing from a base computed once per
+// kernel (the compiler otherwise re-derives the window base per access)
+__device__ __forceinline__ float lds_f32(unsigned a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ unsigned lds_u8(unsigned a) {
+  unsigned v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+#define SMF(off) lds_f32(sbase + 4u * (unsigned)(off))
+#define SMB(off) lds_u8(sbase + (unsigned)(off))
 
 template <int METRIC>
 __device__ __forceinline__ float loc16_dist(const float (&x)[16], const float* __restrict__ m) {
@@ -2285,6 +2385,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
                                               long long* __restrict__ cnt,
                                               const double* __restrict__ scale_s, long long& nfb) {
   extern __shared__ __align__(16) unsigned char smraw[];
+  const unsigned sbase = smem_u32(smraw);
   constexpr int PPT = LOC16_PPT;
   static_assert(PPT == 1, "x[] holds the coordinates of one point per lane");
   const int lane = threadIdx.x & 31, c0 = (threadIdx.x >> 5) * 32 * PPT, d = p.d;
@@ -2301,7 +2402,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
   RingPos rp;
   for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
     const int stg = rp.stg;
-    mbar_wait(&R.full[stg], rp.ph);
+    mbar_wait(R.full_a + 8u * stg, rp.ph);
     const int xs = buf_f + stg * sstride;  // stage base (floats)
     const int xq = xs + c0 + lane;         // lane's first point, row 0
     const int xr = xs + j * LD + c0;       // (h, j) view; j >= d: unused rows
@@ -2313,6 +2414,9 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
         x[jj] = jj < d ? v : 0.f;
       }
     }
+#ifdef LOC_NOP
+    if (na > 0) { pipe_release(R, stg); continue; }  // timing experiment only
+#endif
     for (int a = 0; a < na; ++a) {
       const int rs = row_s[a];
       const Thr t = thr_s[a];
@@ -2370,7 +2474,10 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
 // One point per lane; the cached Dist rows of the active slots arrive through
 // the same TMA ring as the data (rows d..).  DR: coordinates in registers.
 template <int DR>
-__global__ void __launch_bounds__(288, 3) k_locality(RunParams p) {
+#ifndef LOC_MINB
+#define LOC_MINB 3
+#endif
+__global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
   DevState* st = p.st;
   if (st->done) return;
   extern __shared__ __align__(16) unsigned char smraw[];
@@ -2448,7 +2555,7 @@ __global__ void __launch_bounds__(288, 3) k_locality(RunParams p) {
       RingPos rp;
       for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
         const int stg = rp.stg;
-        mbar_wait(&R.full[stg], rp.ph);
+        mbar_wait(R.full_a + 8u * stg, rp.ph);
         const float* xs = R.buf + (size_t)stg * R.rows * LD;
         const bool valid = gp < p.n;
         float xr[DR > 0 ? DR : 1];
@@ -2729,7 +2836,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     RingPos rp;
     for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
       const int stg = rp.stg;
-      mbar_wait(&R.full[stg], rp.ph);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const float* xq = xs + q0 + (IL ? 2 * lane : lane);
       float best[PPT], second[PPT];
@@ -2880,7 +2987,7 @@ __global__ void __launch_bounds__(288) k_labelsum(RunParams p) {
     RingPos rp;
     for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
       const int stg = rp.stg;
-      mbar_wait(&R.full[stg], rp.ph);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const int lb = gp < p.n ? (int)R.lab[(size_t)stg * P + q] : -1;
       // one ballot per cluster: lane c of the warp keeps cluster c's mask
@@ -2938,19 +3045,19 @@ __device__ void pipe_produce_k(const RunParams& p, const Pipe& R, const SmemLayo
   int stg = 0, round = 0;
   for (long long i = 0; i < nmy; ++i) {
     if (round > 0) {
-      mbar_wait(&R.empty[stg], (unsigned)((round - 1) & 1));
+      mbar_wait(R.empty_a + 8u * stg, (unsigned)((round - 1) & 1));
       fence_proxy_async();
     }
     const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
     const long long left = p.n_pad - base;
     const unsigned cnt = (unsigned)(left < P ? left : P);
     const unsigned bytes = cnt * 4u * (unsigned)d + (labsrc ? cnt : 0u);
-    if (lane == 0) mbar_expect_tx(&R.full[stg], bytes);
+    if (lane == 0) mbar_expect_tx(R.full_a + 8u * stg, bytes);
     __syncwarp();
     float* dst = R.buf + (size_t)stg * d * L.ldr;
     for (int j = lane; j < d; j += 32)
-      bulk_g2s(dst + (size_t)j * L.ldr, p.xs + (size_t)j * p.n_pad + base, cnt * 4u, &R.full[stg]);
-    if (labsrc && lane == 0) bulk_g2s(R.lab + (size_t)stg * P, labsrc + base, cnt, &R.full[stg]);
+      bulk_g2s(dst + (size_t)j * L.ldr, p.xs + (size_t)j * p.n_pad + base, cnt * 4u, R.full_a + 8u * stg);
+    if (labsrc && lane == 0) bulk_g2s(R.lab + (size_t)stg * P, labsrc + base, cnt, R.full_a + 8u * stg);
     if (++stg == L.stages) {
       stg = 0;
       ++round;
@@ -3256,7 +3363,7 @@ __global__ void __launch_bounds__(416) k_lsum2(RunParams p) {
       int* hist = X.hist0 + hb * KMAX;
       int* base_s = X.hist0 + 2 * KMAX + hb * KMAX;
       int* list = X.list0 + hb * P;
-      mbar_wait(&R.full[stg], rp.ph);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
       sort_chunk(R.lab + (size_t)stg * P, p.n - g0, q, nct, k, hist, X.hist0 + (hb ^ 1) * KMAX,
                  base_s, list);
       items_chunk<REF ? 1 : 0>(X, reinterpret_cast<const char*>(R.buf + (size_t)stg * d * L.ldr),
@@ -3351,7 +3458,7 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
     RingPos rp;
     for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
       const int stg = rp.stg;
-      mbar_wait(&R.full[stg], rp.ph);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
       if (gp < p.n) {
         const int c = R.lab[(size_t)stg * P + q];
         const char* xq = reinterpret_cast<const char*>(R.buf + (size_t)stg * R.rows * R.ldr + q);
@@ -3444,7 +3551,7 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
     for (long long i = 0; i < nmy; ++i, rp.next(p.stages)) {
       const int stg = rp.stg;
       const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
-      mbar_wait(&R.full[stg], rp.ph);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
 #pragma unroll
       for (int u = 0; u < PPT; ++u) {
