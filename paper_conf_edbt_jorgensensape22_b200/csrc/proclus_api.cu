@@ -368,8 +368,9 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
       e = std::min(e, 50 - (int)std::ceil(std::log2(2.0 * (double)m)));
       e = std::max(-1000, std::min(1000, e));
     }
-    // a sum of <= 32 terms (<= 64 max|x_j|) below 2^51: quant_sum's fma path
-    if (m > 0.f && std::ldexp(64.0 * (double)m, e) >= std::ldexp(1.0, 51)) h->qmagic = 0;
+    // a band sum of <= 256 terms (<= 512 max|x_j|, one chunk of the wide
+    // locality consumer) below 2^51: quant_sum's fma path
+    if (m > 0.f && std::ldexp(512.0 * (double)m, e) >= std::ldexp(1.0, 51)) h->qmagic = 0;
     sc[(size_t)j] = std::ldexp(1.0, e);
     isc[(size_t)j] = std::ldexp(1.0, -e);
   }

@@ -2222,85 +2222,6 @@ __device__ __forceinline__ Thr make_thr(double lo, double hi, double G) {
   return t;
 }
 
-// Band sums of eq 6 for d <= 16, one lane per (half-warp h, dimension j):
-// both half-warps walk the same member mask of slot a (half h takes the
-// members at even / odd positions), so every lane of the warp does the same
-// number of visits whatever the band sizes (the lane-per-cell walk of
-// warp_cells is as slow as its largest cell).  Each visit reads one point's
-// d coordinates across the lanes of a half (rows padded to LD = P + 4: at
-// most 2-way bank conflicts).  fp64 sums of the exact fp64 terms
-// |x_j - m_aj|, combined over the two halves, quantised to int64 at 2^e_j
-// per (slot, dimension, 32-point sub-chunk) exactly as warp_cells does.
-__device__ __forceinline__ void band_sums_d16(const float* __restrict__ xs, int LD, int q0,
-                                              const float* __restrict__ med_s, int MS, int na,
-                                              int d, const unsigned* __restrict__ bal,
-                                              long long* __restrict__ acc,
-                                              const double* __restrict__ scale_s) {
-  const int lane = threadIdx.x & 31, h = lane >> 4, j = lane & 15;
-  const bool jv = j < d;
-  const float* xr = xs + (size_t)(jv ? j : 0) * LD + q0;
-  const double sc = scale_s[jv ? j : 0];
-  for (int a = 0; a < na; ++a) {
-    unsigned m = bal[a];
-    if (h) m &= m - 1u;  // half 1 starts at the second member
-    const double c = (double)med_s[a * MS + (jv ? j : 0)];
-    double s0 = 0.0, s1 = 0.0;
-    while (m) {
-      const int b0 = __ffs(m) - 1;
-      m &= m - 1u;
-      m &= m - 1u;
-      const float x0 = xr[b0];
-      if (m) {
-        const int b1 = __ffs(m) - 1;
-        m &= m - 1u;
-        m &= m - 1u;
-        const float x1 = xr[b1];
-        s1 = dadd(s1, fabs(dsub((double)x1, c)));
-      }
-      s0 = dadd(s0, fabs(dsub((double)x0, c)));
-    }
-    double s = dadd(s0, s1);
-    s = dadd(s, __shfl_xor_sync(0xffffffffu, s, 16));
-    if (h == 0 && jv && s != 0.0) acc[a * d + j] += __double2ll_rn(dmul(s, sc));
-  }
-}
-
-// The same for d > 16: lane = dimension jb + lane of each 32-dimension block,
-// every lane walks the whole member mask of the slot (4-way bank conflicts
-// at the LD = P + 4 row stride instead of 32-way).
-__device__ __forceinline__ void band_sums_gen(const float* __restrict__ xs, int LD, int q0,
-                                              const float* __restrict__ med_s, int MS, int na,
-                                              int d, const unsigned* __restrict__ bal,
-                                              long long* __restrict__ acc,
-                                              const double* __restrict__ scale_s) {
-  const int lane = threadIdx.x & 31;
-  for (int jb = 0; jb < d; jb += 32) {
-    const int j = jb + lane;
-    const bool jv = j < d;
-    const float* xr = xs + (size_t)(jv ? j : 0) * LD + q0;
-    const double sc = scale_s[jv ? j : 0];
-    for (int a = 0; a < na; ++a) {
-      unsigned m = bal[a];
-      const double c = (double)med_s[a * MS + (jv ? j : 0)];
-      double s0 = 0.0, s1 = 0.0;
-      while (m) {
-        const int b0 = __ffs(m) - 1;
-        m &= m - 1u;
-        const float x0 = xr[b0];
-        if (m) {
-          const int b1 = __ffs(m) - 1;
-          m &= m - 1u;
-          const float x1 = xr[b1];
-          s1 = dadd(s1, fabs(dsub((double)x1, c)));
-        }
-        s0 = dadd(s0, fabs(dsub((double)x0, c)));
-      }
-      const double s = dadd(s0, s1);
-      if (jv && s != 0.0) acc[a * d + j] += __double2ll_rn(dmul(s, sc));
-    }
-  }
-}
-
 // Fixed-point quantisation round(s * 2^e_j) of a band / cell sum.  With
 // |s 2^e_j| < 2^51 (p.qmagic, checked on the host for every dimension) one
 // fma with 1.5 * 2^52 rounds to the integer grid exactly as __double2ll_rn
@@ -2470,6 +2391,125 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
 #undef SMF
 #undef SMB
 
+// --- k_locality consumer for d > 16 (wide rows; C4: d = 100).  The LOCW_NW
+// consumer warps share every chunk of P points instead of owning 32 points
+// each (at long rows a chunk is short, P = 64, and per-warp point ownership
+// left 2 consumer warps per block).  Phase A, items (slot a, point block pb
+// of 32 points): lane = point; the certified fp32 distance (computed from
+// the ring for a new Dist row, else read from the cached row), a ballot, and
+// the member's rank compact the members of (a, pb) into a byte list of the
+// ring stage.  Consumer barrier.  Phase B, items (slot a, dimension block jb
+// of 32): lane = dimension j = 32 jb + lane; fp64 sum of the exact terms
+// |x_j - m_aj| over the members of slot a in ascending point order (two
+// interleaved accumulators), quantised per (slot, dimension, chunk) into the
+// block's single accumulator copy: the item -> warp map is fixed within a
+// launch, so every cell has one writer.  A chunk (P | 1024 points, aligned)
+// is one quantisation group, so the totals do not depend on the grid or on
+// 1024-aligned shard boundaries.
+constexpr int LOCW_NW = 8;
+
+template <int METRIC>
+__device__ __forceinline__ void locw_consume(const RunParams& p, const Pipe& R, long long nmy,
+                                             int na, const float* __restrict__ med_s, int MS,
+                                             const int* __restrict__ row_s,
+                                             const Thr* __restrict__ thr_s,
+                                             const ActSlot* __restrict__ act_s,
+                                             unsigned char* __restrict__ lst_s,
+                                             int* __restrict__ lcnt_s,
+                                             long long* __restrict__ acc,
+                                             long long* __restrict__ cnt,
+                                             const double* __restrict__ scale_s, long long& nfb) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, d = p.d, P = p.P, LD = R.ldr;
+  const int npb = P >> 5, nb = (d + 31) >> 5;
+  const int nA = na * npb, nB = na * nb;
+  const int magic = p.qmagic, variant = p.variant;
+  const unsigned lt = (1u << lane) - 1u;
+  const long long n = p.n, n_pad = p.n_pad;
+  long long base = (long long)blockIdx.x * P;
+  const long long gstep = (long long)gridDim.x * P;
+  RingPos rp;
+  for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
+    const int stg = rp.stg;
+    mbar_wait(R.full_a + 8u * stg, rp.ph);
+    const float* xs = R.buf + (size_t)stg * R.rows * LD;
+    unsigned char* lst = lst_s + (size_t)stg * KMAX * P;
+    int* lcnt = lcnt_s + stg * KMAX * 8;
+    for (int it = w; it < nA; it += LOCW_NW) {  // phase A: band decisions
+      const int a = it / npb, pb = it - a * npb;
+      const int q = pb * 32 + lane;
+      const long long gp = base + q;
+      const bool valid = gp < n;
+      const int rs = row_s[a];
+      float f;
+      if (rs < 0) {  // a new Dist row, two fp32 chains
+        const float* m = med_s + a * MS;
+        const float* xq = xs + q;
+        float s0 = 0.f, s1 = 0.f;
+        int j = 0;
+        for (; j + 2 <= d; j += 2) {
+          const float t0 = xq[j * LD] - m[j], t1 = xq[(j + 1) * LD] - m[j + 1];
+          if (METRIC == 1) {
+            s0 = s0 + fabsf(t0);
+            s1 = s1 + fabsf(t1);
+          } else {
+            s0 = __fmaf_rn(t0, t0, s0);
+            s1 = __fmaf_rn(t1, t1, s1);
+          }
+        }
+        if (j < d) {
+          const float t0 = xq[j * LD] - m[j];
+          s0 = METRIC == 1 ? s0 + fabsf(t0) : __fmaf_rn(t0, t0, s0);
+        }
+        f = METRIC == 1 ? s0 + s1 : sqrtf(s0 + s1);
+        if (variant != 1 && valid) p.dist[(long long)act_s[a].key * n_pad + gp] = f;
+      } else {
+        f = xs[rs + q];
+      }
+      const Thr t = thr_s[a];
+      bool in = f < t.in_hi && f > t.out_lo;
+      if (valid && !in && !(f > t.out_hi || f < t.in_lo)) {
+        // within the fp32 error bound: the oracle's fp64 value decides
+        const ActSlot A = act_s[a];
+        const double dv = full_dist(xs + q, LD, med_s + a * MS, d, METRIC);
+        in = (dv > A.lo) && (dv <= A.hi);
+        ++nfb;
+      }
+      in = in && valid;
+      const unsigned b = __ballot_sync(0xffffffffu, in);
+      if (in) lst[a * P + pb * 32 + __popc(b & lt)] = (unsigned char)lane;
+      if (lane == 0) {
+        lcnt[a * 8 + pb] = __popc(b);
+        cnt[w * KMAX + a] += __popc(b);
+      }
+    }
+    named_bar_sync(1, LOCW_NW * 32);  // every (slot, point block) list of the chunk is written
+    for (int it = w; it < nB; it += LOCW_NW) {  // phase B: band sums of eq 6
+      const int a = it / nb, jb = it - a * nb;
+      const int j = jb * 32 + lane;
+      const bool jv = j < d;
+      const float* xr = xs + (size_t)(jv ? j : 0) * LD;
+      const double c = (double)med_s[a * MS + (jv ? j : 0)];
+      double s0 = 0.0, s1 = 0.0;
+      for (int pb = 0; pb < npb; ++pb) {
+        const int m = lcnt[a * 8 + pb];
+        const unsigned char* la = lst + a * P + pb * 32;
+        const float* xb = xr + pb * 32;
+        int v = 0;
+        for (; v + 2 <= m; v += 2) {
+          const double t0 = fabs(dsub((double)xb[la[v]], c));
+          const double t1 = fabs(dsub((double)xb[la[v + 1]], c));
+          s0 = dadd(s0, t0);
+          s1 = dadd(s1, t1);
+        }
+        if (v < m) s0 = dadd(s0, fabs(dsub((double)xb[la[v]], c)));
+      }
+      const double s = dadd(s0, s1);
+      if (jv && s != 0.0) acc[a * d + j] += quant_sum(s, scale_s[j], magic);
+    }
+    pipe_release(R, stg);
+  }
+}
+
 // --- ComputeL + FindDimensions X (Alg 3, Alg 4 l.1-5) with the FAST caches.
 // One point per lane; the cached Dist rows of the active slots arrive through
 // the same TMA ring as the data (rows d..).  DR: coordinates in registers.
@@ -2483,17 +2523,15 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
   extern __shared__ __align__(16) unsigned char smraw[];
   const SmemLayout& L = p.lay[KK_LOC];
 #define LAYK KK_LOC
-  const int P = p.P, d = p.d, k = p.k;
-  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5;
   const int na = st->n_act;
   const int ncap = k * d;
   const Pipe R = pipe_of(L, smraw, DR == 16 && d + k < 16 ? 16 : d + k);
-  const int LD = R.ldr;
   float* med_s = SMP(float, med);
   ActSlot* act_s = SMP(ActSlot, act);
   int* row_s = SMP(int, row);
   double* scale_s = SMP(double, scale);
-  unsigned* bal_s = SMP(unsigned, bal);
   long long* acc_s = SMP(long long, acc);
   long long* cnt_s = SMP(long long, cnt);
   ExtraRows* ex = SMP(ExtraRows, ex);
@@ -2507,7 +2545,7 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
     thr_s[a] = make_thr(st->act[a].lo, st->act[a].hi, G);
   }
   for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
-  for (int e = threadIdx.x; e < nw * ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < (DR == 16 ? nw : 1) * ncap; e += blockDim.x) acc_s[e] = 0;
   for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
   pipe_init(p, R, nw);
   __syncthreads();
@@ -2546,89 +2584,18 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
                          L.tab + w * 32 * LOC16_PPT, acc_s + (size_t)w * ncap, cnt_s + w * KMAX, scale_s,
                          nfb);
     } else {
-      unsigned* bal = bal_s + w * KMAX;
-      long long* acc = acc_s + (size_t)w * ncap;
-      const int q = w * 32 + lane;
-      const int metric = p.metric;
-      long long gp = (long long)blockIdx.x * P + q;
-      const long long gstep = (long long)gridDim.x * P;
-      RingPos rp;
-      for (long long i = 0; i < nmy; ++i, gp += gstep, rp.next(p.stages)) {
-        const int stg = rp.stg;
-        mbar_wait(R.full_a + 8u * stg, rp.ph);
-        const float* xs = R.buf + (size_t)stg * R.rows * LD;
-        const bool valid = gp < p.n;
-        float xr[DR > 0 ? DR : 1];
-        if (DR > 0 && ncomp > 0) {  // coordinates only when a Dist row is computed
-#pragma unroll
-          for (int j = 0; j < DR; ++j) xr[j] = (j < d) ? xs[j * LD + q] : 0.f;
-        }
-        for (int a = 0; a < na; ++a) {
-          const int rs = row_s[a];
-          bool in = false;
-          if (valid) {
-            float f;
-            if (rs < 0) {  // compute distances only once
-              const float* m = med_s + a * MS;
-              float s = 0.f;
-              if (DR > 0) {  // padded coordinates are 0 on both sides
-                const float4* m4 = reinterpret_cast<const float4*>(m);
-                if (metric == 1) {
-#pragma unroll
-                  for (int j4 = 0; j4 < MSD / 4; ++j4) {
-                    const float4 v = m4[j4];
-                    s += fabsf(xr[4 * j4] - v.x) + fabsf(xr[4 * j4 + 1] - v.y) +
-                         fabsf(xr[4 * j4 + 2] - v.z) + fabsf(xr[4 * j4 + 3] - v.w);
-                  }
-                } else {
-                  float s1 = 0.f;
-#pragma unroll
-                  for (int j4 = 0; j4 < MSD / 4; ++j4) {
-                    const float4 v = m4[j4];
-                    const float t0 = xr[4 * j4] - v.x, t1 = xr[4 * j4 + 1] - v.y;
-                    const float t2 = xr[4 * j4 + 2] - v.z, t3 = xr[4 * j4 + 3] - v.w;
-                    s = fmaf(t0, t0, s);
-                    s1 = fmaf(t1, t1, s1);
-                    s = fmaf(t2, t2, s);
-                    s1 = fmaf(t3, t3, s1);
-                  }
-                  s = sqrtf(s + s1);
-                }
-              } else {
-                s = approx_full(xs + q, LD, m, d, metric);
-              }
-              f = s;
-              if (p.variant != 1) p.dist[(long long)act_s[a].key * p.n_pad + gp] = f;
-            } else {
-              f = xs[rs + q];
-            }
-            const Thr t = thr_s[a];
-            if (f < t.in_hi && f > t.out_lo) {
-              in = true;
-            } else if (f > t.out_hi || f < t.in_lo) {
-              in = false;
-            } else {  // within the fp32 error bound: the oracle's fp64 value
-              const ActSlot A = act_s[a];
-              const double dv = full_dist(xs + q, LD, med_s + a * MS, d, metric);
-              in = (dv > A.lo) && (dv <= A.hi);
-              ++nfb;
-            }
-          }
-          put_ballot(bal, a, in);
-        }
-        __syncwarp();
-        if (lane < na) cnt_s[w * KMAX + lane] += __popc(bal[lane]);
-        // cells (a, j): band sum of |x_j - m_aj| (eq 6)
-        if (DR == 16)
-          band_sums_d16(xs, LD, w * 32, med_s, MS, na, d, bal, acc, scale_s);
-        else
-          band_sums_gen(xs, LD, w * 32, med_s, MS, na, d, bal, acc, scale_s);
-        pipe_release(R, stg);
-      }
+      unsigned char* lst_s = SMP(unsigned char, tab);  // [stages][KMAX][P] member lists
+      int* lcnt_s = SMP(int, dl);                      // [stages][KMAX][8] list lengths
+      if (p.metric == 1)
+        locw_consume<1>(p, R, nmy, na, med_s, MS, row_s, thr_s, act_s, lst_s, lcnt_s, acc_s,
+                        cnt_s, scale_s, nfb);
+      else
+        locw_consume<0>(p, R, nmy, na, med_s, MS, row_s, thr_s, act_s, lst_s, lcnt_s, acc_s,
+                        cnt_s, scale_s, nfb);
     }
   }
   __syncthreads();
-  flush_warps(p, acc_s, nw, ncap, na * d, cnt_s, na);
+  flush_warps(p, acc_s, nw, ncap, na * d, cnt_s, na, DR == 16 ? nw : 1);
   if (nfb) atomicAdd((unsigned long long*)&st->fallback[0], (unsigned long long)nfb);
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[0])) return;
@@ -3703,7 +3670,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   const int ppt2 = P >= 128 ? 2 : 1;
   const int nw1 = P / 32, nw2 = P / (32 * ppt2);
   ps.ppt2 = ppt2;
-  ps.tpb_loc = 32 * ((d <= 16 ? nw1 / LOC16_PPT : nw1) + 1);
+  ps.tpb_loc = 32 * ((d <= 16 ? nw1 / LOC16_PPT : LOCW_NW) + 1);
   ps.tpb_asg = 32 * (nw2 + 1);  // updated below when assign takes 2 P
   ps.tpb_lsum = 32 * (nw1 + 1);
   ps.tpb_fin = 32 * (nw2 + 1);
@@ -3713,8 +3680,10 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   {  // locality
     SmemLayout L = blank_layout();
     LB b;
-    // d <= 16: LOC16_PPT points per lane (k_locality<16>), fewer consumer warps
-    L.nw = d <= 16 ? nw1 / LOC16_PPT : nw1;
+    // d <= 16: LOC16_PPT points per lane (k_locality<16>); d > 16: LOCW_NW
+    // consumer warps share each chunk (locw_consume)
+    const int nwl = d <= 16 ? nw1 / LOC16_PPT : LOCW_NW;
+    L.nw = nwl;
     L.P = P;
     // rows padded by 4 floats so that the lane-per-dimension band sums of
     // k_locality read a point's coordinates with at most 2- (d <= 16) or
@@ -3728,14 +3697,17 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.act = b.take(sizeof(ActSlot) * KMAX);
     L.row = b.take(4 * KMAX);
     L.scale = b.take(8 * (size_t)d);
-    L.bal = b.take(4 * (size_t)nw1 * KMAX);
-    L.acc = b.take(8 * (size_t)nw1 * kd);
-    L.cnt = b.take(8 * (size_t)nw1 * KMAX);
+    L.bal = b.take(4 * (size_t)nwl * KMAX);
+    L.acc = b.take(8 * (size_t)(d <= 16 ? nwl : 1) * kd);  // wide: one shared copy
+    L.cnt = b.take(8 * (size_t)nwl * KMAX);
     L.ex = b.take(sizeof(ExtraRows));
     L.thr = b.take(sizeof(Thr) * KMAX);
     if (d <= 16) {
       L.ctr = b.take(8 * (size_t)k * 16);        // fp64 medoid rows of the d <= 16 consumer
       L.tab = b.take((size_t)nw1 * 32);          // per-warp member lists (32 PPT points)
+    } else {
+      L.tab = b.take((size_t)stages * KMAX * P);  // per-stage member lists of (slot, block)
+      L.dl = b.take(4 * (size_t)stages * KMAX * 8);  // their lengths (P <= 256: 8 blocks)
     }
     finish(L, b, ps.tl);
     ps.lay[KK_LOC] = L;
