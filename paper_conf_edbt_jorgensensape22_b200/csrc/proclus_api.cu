@@ -874,7 +874,9 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   // of their own (the north_star's separate Z-score / selection kernel)
   // instead of the last block of each pass; graph mode still applies
   const char* tk_env = getenv("PROCLUS_TAIL_KERNELS");
-  const bool tail_kernels = h->world == 1 && tk_env && tk_env[0] == '1';
+  const bool tail_kernels =
+      h->world == 1 && (ps.split_tails || (tk_env && tk_env[0] == '1')) &&
+      !(tk_env && tk_env[0] == '0');
   p.fuse_tail = (h->world == 1 && !force_split && !tail_kernels) ? 1 : 0;
   p.cost1 = ps.cost1;
   p.qmagic = h->qmagic;

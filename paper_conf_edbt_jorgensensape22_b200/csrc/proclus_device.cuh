@@ -9,7 +9,7 @@
 namespace pc {
 
 constexpr int KMAX = 32;    // k <= 32: per-point medoid membership is a u32
-constexpr int TPB_MAX = 512;
+constexpr int TPB_MAX = 1024;  // threads of the standalone tail kernels
 constexpr int WMAX = 8;     // warps per pass block
 constexpr int UMAX = 4;     // points per thread in a chunk
 constexpr int SMAX = 3;     // max bulk-copy ring depth

@@ -1609,18 +1609,24 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
       if (r0 + r1 < R) dm[c] = 1;
     }
   } else if (R > 0) {
+    // k d > 512: most-significant-digit radix select (8-bit digits) of the R
+    // smallest free keys; as soon as the bucket that holds the R-th key has
+    // at most bd members it is finished by an exact (key, cell) rank among
+    // its members.  Cells below the bucket's prefix are selected.
     __shared__ unsigned int hist[256];
     __shared__ unsigned long long prefix_s;
-    __shared__ int need_s;
-    __shared__ int tcount[TPB_MAX];
+    __shared__ int need_s, bsize_s, bcnt_s;
+    int* blist = reinterpret_cast<int*>(T.Z);  // [<= bd] bucket members (Z is dead here)
     if (tid == 0) {
       prefix_s = 0ull;
       need_s = R;
+      bsize_s = kd;
     }
     unsigned long long hmask = 0ull;
     for (int shift = 56; shift >= 0; shift -= 8) {
-      for (int b = tid; b < 256; b += bd) hist[b] = 0u;
+      for (int bb = tid; bb < 256; bb += bd) hist[bb] = 0u;
       __syncthreads();
+      if (bsize_s <= bd) break;  // small bucket: exact rank below
       const unsigned long long pre = prefix_s;
       for (int c = tid; c < kd; c += bd) {
         if (dm[c]) continue;
@@ -1631,9 +1637,9 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
       if (tid < 32) {  // warp scan over 256 bins, 8 per lane
         unsigned loc[8], tot = 0;
 #pragma unroll
-        for (int b = 0; b < 8; ++b) {
-          loc[b] = hist[tid * 8 + b];
-          tot += loc[b];
+        for (int q = 0; q < 8; ++q) {
+          loc[q] = hist[tid * 8 + q];
+          tot += loc[q];
         }
         unsigned x = tot;
 #pragma unroll
@@ -1648,48 +1654,48 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
         const unsigned who = __ballot_sync(0xffffffffu, here);
         if (here && tid == __ffs(who) - 1) {
           unsigned cum = before;
-          int b = 0;
-          for (; b < 8; ++b) {
-            if ((int)(cum + loc[b]) >= need) break;
-            cum += loc[b];
+          int q = 0;
+          for (; q < 8; ++q) {
+            if ((int)(cum + loc[q]) >= need) break;
+            cum += loc[q];
           }
           need_s = need - (int)cum;
-          prefix_s = pre | ((unsigned long long)(tid * 8 + b) << shift);
+          bsize_s = (int)loc[q];
+          prefix_s = pre | ((unsigned long long)(tid * 8 + q) << shift);
         }
       }
       hmask |= 255ull << shift;
       __syncthreads();
     }
-    const unsigned long long K = prefix_s;
-    const int need = need_s;  // how many cells with key == K to take, in (i, j) order
-    const int per = (kd + bd - 1) / bd;
-    const int c0 = tid * per, c1 = min(kd, c0 + per);
-    int eq = 0;
-    for (int c = c0; c < c1; ++c)
-      if (!dm[c] && key[c] == K) ++eq;
-    tcount[tid] = eq;
+    // bucket = free cells whose decided digits equal the prefix; below it: selected
+    const unsigned long long pre = prefix_s;
+    if (tid == 0) bcnt_s = 0;
     __syncthreads();
-    if (tid < 32) {  // exclusive scan of tcount[0..bd) by one warp
-      int run = 0;
-      for (int b0 = 0; b0 < bd; b0 += 32) {
-        const int v = (b0 + tid < bd) ? tcount[b0 + tid] : 0;
-        int x = v;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int y = __shfl_up_sync(0xffffffffu, x, o);
-          if (tid >= o) x += y;
-        }
-        if (b0 + tid < bd) tcount[b0 + tid] = run + x - v;
-        run += __shfl_sync(0xffffffffu, x, 31);
+    for (int c = tid; c < kd; c += bd) {
+      if (dm[c]) continue;
+      const unsigned long long kp = key[c] & hmask;
+      if (kp < pre) {
+        dm[c] = 2;  // selected (marked 2 until the bucket is ranked: still "free" there)
+      } else if (kp == pre) {
+        blist[atomicAdd(&bcnt_s, 1)] = c;
       }
     }
     __syncthreads();
-    int rank = tcount[tid];
-    for (int c = c0; c < c1; ++c) {  // own contiguous range only
-      if (dm[c]) continue;
+    const int nb = bcnt_s, need = need_s;
+    for (int t = tid; t < nb; t += bd) {  // exact rank inside the bucket by (key, cell)
+      const int c = blist[t];
       const unsigned long long kc = key[c];
-      if (kc < K || (kc == K && rank++ < need)) dm[c] = 1;
+      int r = 0;
+      for (int o = 0; o < nb; ++o) {
+        const int co = blist[o];
+        const unsigned long long ko = key[co];
+        r += (ko < kc) | ((ko == kc) & (co < c));
+      }
+      if (r < need) dm[c] = 2;
     }
+    __syncthreads();
+    for (int c = tid; c < kd; c += bd)
+      if (dm[c] == 2) dm[c] = 1;
   }
   __syncthreads();
   TST(T, tq < 0 ? 6 : tq);
@@ -1786,7 +1792,7 @@ __device__ void prepare_s(const RunParams& p, TailMem& T) {
   TST(T, 17);
 }
 
-__global__ void k_prepare(RunParams p) {
+__global__ void __launch_bounds__(1024, 1) k_prepare(RunParams p) {
   extern __shared__ __align__(16) unsigned char smraw[];
   TailMem T = tail_mem(p, smraw);
   T.mrow = nullptr;  // first iteration: read M and the tables from global memory
@@ -1797,7 +1803,7 @@ __global__ void k_prepare(RunParams p) {
 }
 
 void launch_prepare(const RunParams& p, cudaStream_t s) {
-  k_prepare<<<1, 256, p.tail_smem, s>>>(p);
+  k_prepare<<<1, 1024, p.tail_smem, s>>>(p);
 }
 
 // ------------------------------------------------------------ per-pass tails
@@ -3570,7 +3576,7 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
 }
 
 // ============================================================ multi-GPU tail
-__global__ void k_tail(RunParams p, int tail) {
+__global__ void __launch_bounds__(1024, 1) k_tail(RunParams p, int tail) {
   extern __shared__ __align__(16) unsigned char smraw[];
   DevState* st = p.st;
   if (tail != TAIL_REF && st->done) return;
@@ -3587,7 +3593,7 @@ __global__ void k_tail(RunParams p, int tail) {
 }
 
 void launch_tail(const RunParams& p, int tail, cudaStream_t s) {
-  k_tail<<<1, 256, p.tail_smem, s>>>(p, tail);
+  k_tail<<<1, 1024, p.tail_smem, s>>>(p, tail);
 }
 
 // ============================================================ shapes
@@ -3643,10 +3649,11 @@ static TailLayout tail_layout(int d, int k, int nM) {
   return t;
 }
 
+static bool g_split_tails = false;  // set by pass_shape before the layouts are built
 static void finish(SmemLayout& L, LB& b, const TailLayout& tl) {
   L.tail = L.buf;
   size_t end = b.off;
-  if ((size_t)L.tail + tl.bytes > end) end = (size_t)L.tail + tl.bytes;
+  if (!g_split_tails && (size_t)L.tail + tl.bytes > end) end = (size_t)L.tail + tl.bytes;
   L.bytes = (int)((end + 64 + 15) & ~(size_t)15);
 }
 
@@ -3677,6 +3684,11 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   const size_t kd = (size_t)k * d;
   ps.tl = tail_layout(d, k, nM);
   ps.tail_smem = ps.tl.bytes;
+  // large k d: the single-block tails (radix selection over k d
+  // cells, k^2 medoid distances) run as 1024-thread kernels of their own, and
+  // the pass kernels do not reserve shared memory for them
+  ps.split_tails = kd > 512 ? 1 : 0;
+  g_split_tails = ps.split_tails != 0;
   {  // locality
     SmemLayout L = blank_layout();
     LB b;

@@ -28,6 +28,7 @@ struct PassShape {
   size_t smem_ls2, smem_ref2;
   TailLayout tl;
   int tail_smem;
+  int split_tails;       // 1: the single-block tails run as kernels of their own (k d > 512)
 };
 
 // N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value;

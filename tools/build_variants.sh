@@ -1,5 +1,5 @@
 # build libproclus variants: tools/build_variants.sh NAME "NVCC FLAGS" [NAME "FLAGS" ...]
-set -e
+set -eo pipefail
 cd "$(dirname "$0")/.."
 while [ $# -ge 2 ]; do
   PROCLUS_NVCC_EXTRA="$2" python -c "from paper_conf_edbt_jorgensensape22_b200 import _build; _build.build(force=True)"
