@@ -154,7 +154,7 @@ struct proclus_handle {
   DBuf<int> flag;
   DBuf<unsigned> colmax;
   DBuf<double> scale, iscale;
-  int qmagic = 0;  // every 32-point band sum stays below 2^51 at its scale (RunParams::qmagic)
+  DBuf<int> qflag;  // device: quant_sum fma flag (RunParams::qflag)
   // init-phase products
   DBuf<long long> sids, mids;
   DBuf<float> srows, mrows;
@@ -324,10 +324,21 @@ static proclus_status pin_ensure(proclus_handle* h, size_t bytes) {
   return PROCLUS_OK;
 }
 
+// Exact ceil(log2 x) for x > 0 from the binary exponent (the device's
+// k_scales uses the same rule, so both load paths give identical scales).
+static int ceil_log2(double x) {
+  int ex;
+  const double f = std::frexp(x, &ex);
+  return f == 0.5 ? ex - 1 : ex;
+}
+
 // N0 pack + per-dimension fixed-point scales.  Cell sums of dimension j are
 // bounded by 2 * n_total * max|x_j| (|x - c| with c inside the column range,
 // or |x|), so e_j = 61 - ceil(log2(bound)) keeps every total below 2^61.
-static proclus_status upload_data(proclus_handle* h, const float* data) {
+// sync = false (proclus_load on one GPU): the scales are computed on the
+// device (k_scales) and nothing waits for the host; a non-finite value makes
+// the next proclus_run return EINVAL (k_prepare stops it at once).
+static proclus_status upload_data(proclus_handle* h, const float* data, bool sync) {
   const size_t bytes = sizeof(float) * (size_t)h->n * h->d;
   const float* src = data;
   if (!h->data_on_device) {
@@ -345,6 +356,12 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
   });
   CK(cudaGetLastError());
   if (h->pack_done) CK(cudaEventRecord(h->pack_done, h->stream));  // staging read
+  h->m_valid = false;  // cached M / Dist rows refer to old data
+  if (!sync && h->world == 1) {
+    launch_scales(h->colmax.p, h->d, h->n_total, h->scale.p, h->iscale.p, h->qflag.p, h->stream);
+    CK(cudaGetLastError());
+    return PROCLUS_OK;
+  }
   TRY(allreduce(h, h->colmax.p, h->d, ncclUint32, ncclMax));
   TRY(allreduce(h, h->flag.p, 1, ncclInt32, ncclMax));
   int bad = 0;
@@ -355,22 +372,21 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
   CK(cudaStreamSynchronize(h->stream));
   if (bad) return fail(PROCLUS_EINVAL, "data contains non-finite values");
   std::vector<double> sc((size_t)h->d), isc((size_t)h->d);
-  h->qmagic = 1;
+  int qmagic = 1;
   for (int j = 0; j < h->d; ++j) {
     float m;
     memcpy(&m, &cm[(size_t)j], sizeof(float));
     int e = 0;
     if (m > 0.f) {
-      const double bound = 2.0 * (double)h->n_total * (double)m;
-      e = 61 - (int)std::ceil(std::log2(bound));
+      e = 61 - ceil_log2(2.0 * (double)h->n_total * (double)m);
       // one term (<= 2 max|x_j|) stays below 2^51: the per-term quantisation
       // of the lane-private passes keeps it in the low mantissa bits of a double
-      e = std::min(e, 50 - (int)std::ceil(std::log2(2.0 * (double)m)));
+      e = std::min(e, 50 - ceil_log2(2.0 * (double)m));
       e = std::max(-1000, std::min(1000, e));
+      // a band sum of <= 256 terms (<= 512 max|x_j|, one chunk of the wide
+      // locality consumer) below 2^51: quant_sum's fma path
+      if (std::ldexp(512.0 * (double)m, e) >= std::ldexp(1.0, 51)) qmagic = 0;
     }
-    // a band sum of <= 256 terms (<= 512 max|x_j|, one chunk of the wide
-    // locality consumer) below 2^51: quant_sum's fma path
-    if (m > 0.f && std::ldexp(512.0 * (double)m, e) >= std::ldexp(1.0, 51)) h->qmagic = 0;
     sc[(size_t)j] = std::ldexp(1.0, e);
     isc[(size_t)j] = std::ldexp(1.0, -e);
   }
@@ -378,8 +394,8 @@ static proclus_status upload_data(proclus_handle* h, const float* data) {
                      h->stream));
   CK(cudaMemcpyAsync(h->iscale.p, isc.data(), sizeof(double) * h->d, cudaMemcpyHostToDevice,
                      h->stream));
+  CK(cudaMemcpyAsync(h->qflag.p, &qmagic, sizeof(int), cudaMemcpyHostToDevice, h->stream));
   CK(cudaStreamSynchronize(h->stream));
-  h->m_valid = false;  // cached M / Dist rows refer to old data
   return PROCLUS_OK;
 }
 
@@ -461,13 +477,14 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
       return cleanup(fail(PROCLUS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
   }
   if (h->xs.ensure((size_t)h->n_pad * d) != cudaSuccess || h->flag.ensure(1) != cudaSuccess ||
+      h->qflag.ensure(1) != cudaSuccess ||
       h->colmax.ensure((size_t)d) != cudaSuccess || h->scale.ensure((size_t)d) != cudaSuccess ||
       h->iscale.ensure((size_t)d) != cudaSuccess)
     return cleanup(
         fail(PROCLUS_ENOMEM, "device allocation of %lld x %d failed", (long long)n, d));
   if (cudaMallocHost(&h->h_st, sizeof(DevState)) != cudaSuccess)
     return cleanup(fail(PROCLUS_ENOMEM, "pinned allocation failed"));
-  if ((st = upload_data(h, data)) != PROCLUS_OK) return cleanup(st);
+  if ((st = upload_data(h, data, true)) != PROCLUS_OK) return cleanup(st);
   *out = h;
   return PROCLUS_OK;
 }
@@ -479,7 +496,7 @@ proclus_status proclus_create(const float* data, int64_t n, int32_t d, proclus_h
 proclus_status proclus_load(proclus_handle* h, const float* data) {
   if (!h || !data) return fail(PROCLUS_EINVAL, "NULL argument");
   TRY(set_device(h));
-  return upload_data(h, data);
+  return upload_data(h, data, false);
 }
 
 proclus_status proclus_prefetch(proclus_handle* h, const float* data) {
@@ -516,6 +533,7 @@ void proclus_destroy(proclus_handle* h) {
   h->xs.release();
   h->staging.release();
   h->flag.release();
+  h->qflag.release();
   h->colmax.release();
   h->scale.release();
   h->iscale.release();
@@ -879,7 +897,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
       !(tk_env && tk_env[0] == '0');
   p.fuse_tail = (h->world == 1 && !force_split && !tail_kernels) ? 1 : 0;
   p.cost1 = ps.cost1;
-  p.qmagic = h->qmagic;
+  p.qflag = h->qflag.p;
+  p.badflag = h->flag.p;
   p.variant = h->variant;
   p.out_labels = h->out_labels.p;
   p.Delta = h->Delta.p;
@@ -956,6 +975,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   }
   CK(cudaStreamSynchronize(h->stream));
   if (out && out->dims) memcpy(out->dims, h->h_pin + sizeof(long long) * h->nM, (size_t)k * d);
+  if (h->h_st->err == ERR_NONFINITE)
+    return fail(PROCLUS_EINVAL, "data contains non-finite values (found by the last load)");
   if (h->h_st->err) return fail(PROCLUS_EINTERNAL, "device reported error %d", h->h_st->err);
   const int T = h->h_st->iterations;
   if (use_graph) h->launches += p.fuse_tail ? 1 + 3 * (int64_t)T + 2 : 1 + 6 * (int64_t)T + 3;

@@ -19,6 +19,8 @@ constexpr int PAD_ALIGN = 1024;  // n_pad multiple; shard boundaries for invaria
 
 // One medoid slot whose locality set changes in this iteration
 // (GPU-FAST-PROCLUS).  The band is (lo, hi]: Theorem 3.1 / eq 3.
+constexpr int ERR_NONFINITE = 7;  // DevState::err: non-finite data (asynchronous load)
+
 struct ActSlot {
   int slot;      // cluster slot i in MCur
   int mpos;      // MIdx_i: position in M: the medoid's row of M
@@ -117,7 +119,8 @@ struct RunParams {
   long long nchunks;
   int fuse_tail;           // 1: last block finalises (single GPU)
   int cost1;               // 1: the cost pass sums per cluster (k_cost1), cells 0..k-1
-  int qmagic;              // 1: 32-term band sums stay below 2^51 at 2^e_j (quant_sum fma path)
+  const int* qflag;        // device: 1 = band sums of <= 256 terms stay below 2^51 at 2^e_j
+  const int* badflag;      // device: 1 = the loaded data has a non-finite value
   int variant;             // proclus_variant: 0 FAST, 1 plain (no caches), 2 FAST*
   int use_cond;            // 1: running inside a graph while-node
   unsigned long long cond; // cudaGraphConditionalHandle

@@ -154,6 +154,42 @@ void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float
   k_pack_soa<<<grid, dim3(32, 8), 0, s>>>(in, n, d, n_pad, xs, bad, colmax);
 }
 
+// Per-dimension fixed-point scales 2^e_j from max |x_j| (colmax, float bits):
+// e_j = 61 - ceil(log2(2 n_total max|x_j|)), at most 50 - ceil(log2(2
+// max|x_j|)), clamped to [-1000, 1000]; ceil(log2 x) is taken exactly from the
+// binary exponent (frexp), so the host path (scales_of in proclus_api.cu)
+// computes the same values.  qflag = 0 if some band sum of <= 256 terms can
+// reach 2^51 at its scale (quant_sum then converts instead of the fma).
+__device__ __forceinline__ int ceil_log2_dev(double x) {
+  int ex;
+  const double f = frexp(x, &ex);
+  return f == 0.5 ? ex - 1 : ex;
+}
+__global__ void k_scales(const unsigned* __restrict__ colmax, int d, long long n_total,
+                         double* __restrict__ scale, double* __restrict__ iscale, int* qflag) {
+  __shared__ int ok;
+  if (threadIdx.x == 0) ok = 1;
+  __syncthreads();
+  for (int j = threadIdx.x; j < d; j += blockDim.x) {
+    const float m = __uint_as_float(colmax[j]);
+    int e = 0;
+    if (m > 0.f) {
+      e = 61 - ceil_log2_dev(2.0 * (double)n_total * (double)m);
+      e = min(e, 50 - ceil_log2_dev(2.0 * (double)m));
+      e = max(-1000, min(1000, e));
+      if (ldexp(512.0 * (double)m, e) >= 2251799813685248.0) atomicAnd(&ok, 0);  // 2^51
+    }
+    scale[j] = ldexp(1.0, e);
+    iscale[j] = ldexp(1.0, -e);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) *qflag = ok;
+}
+void launch_scales(const unsigned* colmax, int d, long long n_total, double* scale,
+                   double* iscale, int* qflag, cudaStream_t s) {
+  k_scales<<<1, 256, 0, s>>>(colmax, d, n_total, scale, iscale, qflag);
+}
+
 // Small host -> device uploads as kernel parameters (no copy-engine work, so
 // they never queue behind a proclus_prefetch transfer of the next dataset).
 struct Blob {
@@ -1798,6 +1834,15 @@ __global__ void __launch_bounds__(1024, 1) k_prepare(RunParams p) {
   T.mrow = nullptr;  // first iteration: read M and the tables from global memory
   TST_START();
   state_load(p, T.S);
+  if (*p.badflag) {  // the last (asynchronous) load found a non-finite value
+    if (threadIdx.x == 0) {
+      T.S->err = ERR_NONFINITE;
+      T.S->done = 1;
+      if (p.use_cond) cudaGraphSetConditional((cudaGraphConditionalHandle)p.cond, 0u);
+    }
+    state_store(p, T.S);
+    return;
+  }
   prepare_s(p, T);
   state_store(p, T.S);
 }
@@ -2229,7 +2274,7 @@ __device__ __forceinline__ Thr make_thr(double lo, double hi, double G) {
 }
 
 // Fixed-point quantisation round(s * 2^e_j) of a band / cell sum.  With
-// |s 2^e_j| < 2^51 (p.qmagic, checked on the host for every dimension) one
+// |s 2^e_j| < 2^51 (*p.qflag, set with the scales for every dimension) one
 // fma with 1.5 * 2^52 rounds to the integer grid exactly as __double2ll_rn
 // (the scale is a power of two, so s * 2^e_j itself is exact), on the fp64
 // pipe instead of the 16/clk/SM conversion pipe.
@@ -2320,7 +2365,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
   const int h = lane >> 4, j = lane & 15;
   const unsigned lt = (1u << lane) - 1u;
   const double sc = scale_s[j < d ? j : 0];
-  const int magic = p.qmagic;
+  const int magic = *p.qflag;
   const int variant = p.variant;
   const long long n = p.n, n_pad = p.n_pad;
   float* const dist = p.dist;
@@ -2428,7 +2473,7 @@ __device__ __forceinline__ void locw_consume(const RunParams& p, const Pipe& R, 
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, d = p.d, P = p.P, LD = R.ldr;
   const int npb = P >> 5, nb = (d + 31) >> 5;
   const int nA = na * npb, nB = na * nb;
-  const int magic = p.qmagic, variant = p.variant;
+  const int magic = *p.qflag, variant = p.variant;
   const unsigned lt = (1u << lane) - 1u;
   const long long n = p.n, n_pad = p.n_pad;
   long long base = (long long)blockIdx.x * P;
@@ -3581,6 +3626,7 @@ __global__ void __launch_bounds__(1024, 1) k_tail(RunParams p, int tail) {
   DevState* st = p.st;
   if (tail != TAIL_REF && st->done) return;
   TailMem T = tail_mem(p, smraw);
+  TST_START();
   if (tail == TAIL_LOC)
     tail_locality(p, T);
   else if (tail == TAIL_ASG)

@@ -35,6 +35,10 @@ struct PassShape {
 // colmax[j] = max(colmax[j], bits of max |x_j|).
 void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
                      unsigned* colmax, cudaStream_t s);
+// 2^e_j, 2^-e_j and the quant_sum fma flag from max |x_j| on the device
+// (the asynchronous load path: no host round trip).
+void launch_scales(const unsigned* colmax, int d, long long n_total, double* scale,
+                   double* iscale, int* qflag, cudaStream_t s);
 // rows of the given (global) ids; rows outside [row_offset, row_offset+n)
 // are zero (they are filled by another rank and summed by the allreduce).
 void launch_gather_rows(const float* xs, long long n_pad, int d, const long long* ids,

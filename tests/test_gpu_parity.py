@@ -439,3 +439,20 @@ def test_L8_oracle_parity(pk, orc, k, l):
     del x
     o = orc.proclus(data, k, l, seed=1, trace=True)
     assert_parity(g, o, gt, o.trace, what=f"L8 k={k} l={l}")
+
+
+def test_async_load_rejects_nonfinite_at_run(pk, orc):
+    """proclus_load is asynchronous on one GPU (scales computed on the device):
+    a non-finite value makes the next run fail with EINVAL; a later load of
+    finite data recovers, with results equal to the oracle's."""
+    d1, _ = synth.config_data("C1", seed=1)
+    bad = d1.copy()
+    bad[123, 4] = np.nan
+    with pk.Proclus(d1) as h:
+        h.load(bad)
+        with pytest.raises(pk.ProclusError) as e:
+            h.run(5, 3, seed=1)
+        assert e.value.status == pk.EINVAL
+        h.load(d1)
+        g = h.run(5, 3, seed=1)
+    assert_parity(g, orc.proclus(d1, 5, 3, seed=1), what="after a rejected load")
