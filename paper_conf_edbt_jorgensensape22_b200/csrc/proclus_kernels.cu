@@ -258,16 +258,6 @@ void launch_gather_m(const float* srows, const long long* sids, const int* spos,
 // points, bits(dist) + 1 otherwise.
 constexpr int GR_TPB = 1024;
 
-__global__ void k_sdist(const float* __restrict__ srows, int nS, int d, int metric,
-                        double* __restrict__ Ds) {
-  const long long tot = (long long)nS * nS;
-  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < tot;
-       e += (long long)gridDim.x * blockDim.x) {
-    const int a = (int)(e / nS), q = (int)(e - (long long)a * nS);
-    Ds[e] = full_dist(srows + (long long)q * d, 1, srows + (long long)a * d, d, metric);
-  }
-}
-
 struct KeyIdx {
   unsigned hi, lo, idx;
 };
@@ -637,71 +627,10 @@ __device__ __forceinline__ unsigned long long dkey(double v) {
   return v >= 0.0 ? (unsigned long long)__double_as_longlong(v) + 1ull : 0ull;
 }
 
-// 256 threads x 16 positions in registers; one barrier per pick: every warp
-// publishes its candidate in a parity-double-buffered slot and then all
-// warps reduce the 8 candidates redundantly.
+// gate of the exact-matrix greedy path: #S <= GM_TPB * GM_PPT = 4096
 constexpr int GM_TPB = 256;
 constexpr int GM_PPT = 16;
-__global__ void __launch_bounds__(GM_TPB)
-    k_greedy(const double* __restrict__ Ds, int nS, int nM, int q0, int* __restrict__ spos,
-             double* __restrict__ pickdist) {
-  __shared__ unsigned whi[2][8], wlo[2][8], widx[2][8];
-  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-  constexpr int nw = GM_TPB / 32;
-  double dreg[GM_PPT];
-#pragma unroll
-  for (int t = 0; t < GM_PPT; ++t) {
-    const int q = tid + t * GM_TPB;
-    dreg[t] = (q < nS && q != q0) ? __ldg(Ds + (long long)q0 * nS + q) : -1.0;
-  }
-  if (tid == 0) {
-    spos[0] = q0;
-    if (pickdist) pickdist[0] = CUDART_INF;
-  }
-  for (int i = 1; i < nM; ++i) {
-    unsigned long long bk = 0ull;
-    unsigned bq = 0xffffffffu;
-#pragma unroll
-    for (int t = 0; t < GM_PPT; ++t) {
-      const unsigned long long key = dkey(dreg[t]);
-      if (key > bk) {  // ascending q: strict > keeps the smaller position
-        bk = key;
-        bq = tid + t * GM_TPB;
-      }
-    }
-    KeyIdx r = warp_argmax((unsigned)(bk >> 32), (unsigned)bk, bq);
-    const int par = i & 1;
-    if (lane == 0) {
-      whi[par][w] = r.hi;
-      wlo[par][w] = r.lo;
-      widx[par][w] = r.idx;
-    }
-    __syncthreads();
-    KeyIdx s = warp_argmax(lane < nw ? whi[par][lane] : 0u, lane < nw ? wlo[par][lane] : 0u,
-                           lane < nw ? widx[par][lane] : 0xffffffffu);
-    const int qs = (int)s.idx;
-    if (tid == 0) {
-      spos[i] = qs;
-      if (pickdist) {
-        unsigned long long kk = ((unsigned long long)s.hi << 32) | s.lo;
-        pickdist[i] = __longlong_as_double((long long)(kk - 1ull));
-      }
-    }
-    const double* row = Ds + (long long)qs * nS;
-#pragma unroll
-    for (int t = 0; t < GM_PPT; ++t) {
-      const int q = tid + t * GM_TPB;
-      if (q == qs) {
-        dreg[t] = -1.0;
-      } else if (dreg[t] >= 0.0) {
-        const double u = __ldg(row + q);
-        if (u < dreg[t]) dreg[t] = u;
-      }
-    }
-  }
-}
 
-// Large samples (#S > 4096): same picks, distances computed on the fly.
 __global__ void __launch_bounds__(GR_TPB)
     k_greedy_big(const float* __restrict__ srows, int nS, int d, int nM, int q0, int metric,
                  double* __restrict__ dist, int* __restrict__ spos, double* __restrict__ pickdist) {
@@ -1006,14 +935,11 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
     const int npc = nS <= per ? 1 : nS <= 2 * per ? 2 : nS <= 4 * per ? 4 : 0;
     const int dp = d <= 8 ? 8 : d <= 16 ? 16 : d <= 32 ? 32 : ((d + 1) / 2) * 2;
     const size_t soa = (size_t)dp * npc * per;  // doubles
-    if (npc && sizeof(double) * soa <= 200 * 1024 && soa <= greedy_scratch_doubles(nS) &&
-        !getenv("PROCLUS_GREEDY_1CTA")) {
+    if (npc && sizeof(double) * soa <= 200 * 1024 && soa <= greedy_scratch_doubles(nS)) {
       k_sample_soa<<<(int)((soa + 255) / 256), 256, 0, s>>>(srows, nS, d, dp, npc * per, scratch);
-      cudaError_t e = npc == 1 ? greedy_cluster_np<1>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
-                      : npc == 2 ? greedy_cluster_np<2>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
-                                 : greedy_cluster_np<4>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s);
-      if (e == cudaSuccess) return cudaSuccess;
-      cudaGetLastError();  // cluster launch unavailable: single-CTA kernels below
+      return npc == 1 ? greedy_cluster_np<1>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
+             : npc == 2 ? greedy_cluster_np<2>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s)
+                        : greedy_cluster_np<4>(scratch, nS, d, dp, nM, q0, metric, spos, pickdist, s);
     }
   }
   const int np = nS <= 256 ? 1 : nS <= 512 ? 2 : nS <= 1024 ? 4 : nS <= 2048 ? 8 : 16;
@@ -1026,31 +952,15 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
       default: return greedy_smem_launch<16>(srows, nS, d, nM, q0, metric, spos, pickdist, s);
     }
   }
-  if (nS <= GM_PPT * GM_TPB) {
-    const long long tot = (long long)nS * nS;
-    int blocks = (int)((tot + 255) / 256);
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    if (blocks < 1) blocks = 1;
-    if (getenv("PROCLUS_SDIST_SIMPLE")) {
-      k_sdist<<<blocks, 256, 0, s>>>(srows, nS, d, metric, scratch);
-    } else {
-      const int nt = (nS + SD_T - 1) / SD_T;
-      k_sdist_tiled<<<nt * (nt + 1) / 2, 256, 0, s>>>(srows, nS, d, metric, scratch);
-    }
+  if (nS <= GM_PPT * GM_TPB) {  // <= 4096: exact matrix, picks in a 16-CTA cluster
+    const int nt = (nS + SD_T - 1) / SD_T;
+    k_sdist_tiled<<<nt * (nt + 1) / 2, 256, 0, s>>>(srows, nS, d, metric, scratch);
     const int per = 16 * GC_TPB;
-    const int npm = nS <= 2 * per ? 2 : nS <= 4 * per ? 4 : nS <= 8 * per ? 8 : 0;
-    if (npm && !getenv("PROCLUS_GREEDY_MAT1")) {
-      cudaError_t e = npm == 2   ? greedy_mat_launch<2>(scratch, nS, nM, q0, spos, pickdist, s)
-                      : npm == 4 ? greedy_mat_launch<4>(scratch, nS, nM, q0, spos, pickdist, s)
-                                 : greedy_mat_launch<8>(scratch, nS, nM, q0, spos, pickdist, s);
-      if (e == cudaSuccess) return cudaSuccess;
-      cudaGetLastError();  // cluster launch unavailable: the single-CTA kernel
-    }
-    k_greedy<<<1, GM_TPB, 0, s>>>(scratch, nS, nM, q0, spos, pickdist);
-  } else {
-    k_greedy_big<<<1, GR_TPB, sizeof(double) * d, s>>>(srows, nS, d, nM, q0, metric, scratch,
-                                                       spos, pickdist);
+    return nS <= 2 * per ? greedy_mat_launch<2>(scratch, nS, nM, q0, spos, pickdist, s)
+                         : greedy_mat_launch<4>(scratch, nS, nM, q0, spos, pickdist, s);
   }
+  k_greedy_big<<<1, GR_TPB, sizeof(double) * d, s>>>(srows, nS, d, nM, q0, metric, scratch,
+                                                     spos, pickdist);
   return cudaGetLastError();
 }
 
@@ -2955,6 +2865,198 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
 #undef LAYK
 }
 
+// --- AssignPoints (Alg 5) + centroid sums for long rows (chunks of P <= 64
+// points): the ASW_NW consumer warps share every chunk instead of owning 32
+// points each (round 1 ran C4 with 4 consumer warps per SM).
+// Phase A, items (32-point block pb, cluster range q): lane = point; the
+//   certified fp32 segmental distances of the clusters of range q (two fp32
+//   chains; the certified bound only needs the number of terms) reduced to
+//   (best, second, argmin) in shared memory.
+// Phase B, one warp per point block: merge the ranges in cluster order
+//   (ties -> the smaller cluster, reading R8), certify against the runner-up
+//   or take the exact fp64 argmin, store the u8 label; per-cluster ballots
+//   give the chunk's member masks.
+// Phase C, cells (cluster c, t < |D_c|) over all consumer threads: fp64 sum
+//   of x_j over the chunk's members of c, quantised per (cell, chunk) into
+//   the block's single accumulator copy (one writer per cell), |C_c| counts.
+constexpr int ASW_NW = 8;
+struct __align__(16) Part {
+  float best, second;
+  int bi, pad;
+};
+__global__ void __launch_bounds__(288) k_assign_w(RunParams p) {
+  DevState* st = p.st;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_ASG];
+#define LAYK KK_ASG
+  const int P = p.P, d = p.d, k = p.k;
+  const int nw = ASW_NW, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ncap = k * d;
+  const Pipe R = pipe_of(L, smraw, d);
+  const int LD = R.ldr;
+  float* med_s = SMP(float, med);     // [k][d] medoid rows (exact fallback)
+  Term* tab_s = SMP(Term, tab);       // [k*l] terms, cluster c from off_s[c]
+  int* dl_s = SMP(int, dl);           // [k][d] dimension lists
+  int* nD_s = SMP(int, nD);
+  int* off_s = SMP(int, off);
+  float* rcp_s = SMP(float, rcp);
+  double* scale_s = SMP(double, scale);
+  Cell* cells = SMP(Cell, cells);     // [k*l]
+  unsigned* msk_s = SMP(unsigned, bal);   // [KMAX][npb] member masks of the chunk
+  long long* acc_s = SMP(long long, acc);  // [k*d] one copy
+  long long* cnt_s = SMP(long long, cnt);  // [nw][KMAX], row 0 used
+  Part* part = SMP(Part, row);             // [nq][P]
+  const long long nmy = chunks_of_block(p);
+  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
+  for (int e = threadIdx.x; e < ncap; e += blockDim.x) acc_s[e] = 0;
+  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  pipe_init(p, R, nw);
+  __syncthreads();
+  if (st->done) return;
+  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    nD_s[i] = st->nD[i];
+    rcp_s[i] = 1.0f / (float)st->nD[i];
+  }
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
+    dl_s[e] = p.dlist[e];
+  }
+  __syncthreads();
+  const int ncell = build_cells(cells, nD_s, k, d, off_s, dl_s, nullptr);  // also off_s
+  for (int e = threadIdx.x; e < ncell; e += blockDim.x) {
+    const Cell C = cells[e];
+    Term t;
+    t.m = med_s[C.a * d + C.j];
+    t.m2 = t.m;
+    t.joff = C.j * LD;  // float offset of row j in a ring stage
+    t.pad = 0;
+    tab_s[e] = t;
+  }
+  int ndmax = 0;
+  for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
+  const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
+  __syncthreads();
+  long long nfb = 0;
+  if (w == nw) {
+    pipe_produce(p, R, nmy, nullptr, nullptr);
+  } else {
+    const int npb = P >> 5, nq = nw / npb;
+    const int magic = *p.qflag;
+    long long base = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
+      const float* xs = R.buf + (size_t)stg * R.rows * LD;
+      {  // phase A: item (pb, q) = warp w
+        const int pb = w % npb, q = w / npb;
+        const int c0 = q * k / nq, c1 = (q + 1) * k / nq;
+        const float* xq = xs + pb * 32 + lane;
+        float best = CUDART_INF_F, second = CUDART_INF_F;
+        int bi = c0;
+        for (int c = c0; c < c1; ++c) {
+          const Term* tb = tab_s + off_s[c];
+          const int nd = nD_s[c];
+          float a0 = 0.f, a1 = 0.f;
+          int t = 0;
+          for (; t + 2 <= nd; t += 2) {
+            const Term e0 = tb[t], e1 = tb[t + 1];
+            a0 += fabsf(xq[e0.joff] - e0.m);
+            a1 += fabsf(xq[e1.joff] - e1.m);
+          }
+          if (t < nd) a0 += fabsf(xq[tb[t].joff] - tb[t].m);
+          const float qv = (a0 + a1) * rcp_s[c];
+          second = qv < best ? best : fminf(second, qv);
+          bi = qv < best ? c : bi;
+          best = fminf(best, qv);
+        }
+        Part pr;
+        pr.best = best;
+        pr.second = second;
+        pr.bi = bi;
+        pr.pad = 0;
+        part[q * P + pb * 32 + lane] = pr;
+      }
+      named_bar_sync(1, nw * 32);
+      if (w < npb) {  // phase B: point block w
+        const int qp = w * 32 + lane;
+        const long long gp = base + qp;
+        float best = CUDART_INF_F, second = CUDART_INF_F;
+        int bi = 0;
+        for (int q = 0; q < nq; ++q) {  // cluster order: the earlier range wins ties
+          const Part pr = part[q * P + qp];
+          if (pr.best < best) {
+            second = fminf(best, fminf(second, pr.second));
+            best = pr.best;
+            bi = pr.bi;
+          } else {
+            second = fminf(second, pr.best);
+          }
+        }
+        int lbl = -1;
+        if (gp < p.n) {
+          const bool certain = (best >= 1e-30f) && (second < 1e30f) &&
+                               ((double)second * (1.0 - G) > (double)best * (1.0 + G));
+          lbl = bi;
+          if (!certain) {
+            lbl = exact_argmin(xs + qp, LD, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
+            ++nfb;
+          }
+          lab[gp] = (unsigned char)lbl;
+        }
+        unsigned mine = 0u;
+        for (int c = 0; c < k; ++c) {
+          const unsigned b = __ballot_sync(0xffffffffu, lbl == c);
+          if (lane == c) mine = b;
+        }
+        if (lane < k) msk_s[lane * npb + w] = mine;
+      }
+      named_bar_sync(1, nw * 32);
+      {  // phase C: centroid cells and counts
+        const int tid = threadIdx.x;
+        for (int ci = tid; ci < ncell; ci += nw * 32) {
+          const Cell C = cells[ci];
+          const float* xr = xs + (size_t)C.j * LD;
+          double s0 = 0.0, s1 = 0.0;
+          for (int pb = 0; pb < npb; ++pb) {
+            unsigned m = msk_s[C.a * npb + pb];
+            const float* xb = xr + pb * 32;
+            while (m) {
+              const int b0 = __ffs(m) - 1;
+              m &= m - 1u;
+              s0 = dadd(s0, (double)xb[b0]);
+              if (m) {
+                const int b1 = __ffs(m) - 1;
+                m &= m - 1u;
+                s1 = dadd(s1, (double)xb[b1]);
+              }
+            }
+          }
+          const double sm = dadd(s0, s1);
+          if (sm != 0.0) acc_s[C.acc] += quant_sum(sm, scale_s[C.j], magic);
+        }
+        if (tid < k) {
+          int cn = 0;
+          for (int pb = 0; pb < npb; ++pb) cn += __popc(msk_s[tid * npb + pb]);
+          cnt_s[tid] += cn;
+        }
+      }
+      pipe_release(R, stg);
+      named_bar_sync(1, nw * 32);  // masks and parts are rewritten by the next chunk
+    }
+  }
+  __syncthreads();
+  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, k, 1);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[1])) return;
+  RUN_TAIL(tail_assign, 1);
+#undef LAYK
+}
+
 // --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) + control tail, and the
 // refinement X over CBest (Alg 1 l.16-17) which has the same shape.
 // REF = 0: cells (i, t) over D_i of |x - mu_i|, labels of the current buffer.
@@ -3705,6 +3807,7 @@ static void finish(SmemLayout& L, LB& b, const TailLayout& tl) {
 
 PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   PassShape ps;
+  memset(&ps, 0, sizeof(ps));  // padding too: the graph cache compares it bytewise
   int P = 256, stages = 3;
   const int cfg[6][2] = {{256, 3}, {256, 2}, {128, 3}, {128, 2}, {64, 3}, {64, 2}};
   for (int c = 0; c < 6; ++c) {
@@ -3712,9 +3815,6 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     stages = cfg[c][1];
     if ((size_t)stages * (d + k) * P * 4 <= 60 * 1024) break;
   }
-#ifdef PROCLUS_STAGES2
-  if (stages > 2) stages = 2;
-#endif
   ps.P = P;
   ps.stages = stages;
   // consumer warps at 1 point per lane (locality, cost, refinement) and at
@@ -3800,12 +3900,32 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   };
   ps.P_asg = P;
   ps.lay[KK_ASG] = asg_layout(P);
-  if (ppt2 == 1 && !getenv("PROCLUS_ASG_P1")) {
-    const SmemLayout L2 = asg_layout(2 * P);
-    if (L2.bytes <= 225 * 1024) {  // the 227 KB opt-in limit less static smem
-      ps.P_asg = 2 * P;
-      ps.lay[KK_ASG] = L2;
-    }
+  ps.asg_w = 0;
+  if (ppt2 == 1) {  // long rows: k_assign_w, ASW_NW consumer warps share a chunk
+    SmemLayout L = blank_layout();
+    LB b;
+    const int kl = k * l;
+    L.nw = ASW_NW;
+    L.P = P;
+    L.ldr = P + 4;  // phase C lanes read different rows of one column: <= 4-way conflicts
+    L.full = b.take(8 * SMAX);
+    L.empty = b.take(8 * SMAX);
+    L.buf = b.take((size_t)stages * d * L.ldr * 4);
+    L.med = b.take(4 * kd);
+    L.tab = b.take(sizeof(Term) * (size_t)kl);
+    L.dl = b.take(4 * kd);
+    L.nD = b.take(4 * KMAX);
+    L.off = b.take(4 * (KMAX + 1));
+    L.rcp = b.take(4 * KMAX);
+    L.scale = b.take(8 * (size_t)d);
+    L.cells = b.take(sizeof(Cell) * (size_t)kl);
+    L.bal = b.take(4 * (size_t)KMAX * (P / 32));
+    L.acc = b.take(8 * kd);
+    L.cnt = b.take(8 * (size_t)ASW_NW * KMAX);
+    L.row = b.take(sizeof(Part) * (size_t)(ASW_NW / (P / 32)) * P);
+    finish(L, b, ps.tl);
+    ps.lay[KK_ASG] = L;
+    ps.asg_w = 1;
   }
   {  // labelsum (cost / refinement X)
     SmemLayout L = blank_layout();
@@ -3886,14 +4006,14 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   {
     int nw = 0;
     ps.lay[KK_LS2] = ls2_layout(k * l, nw, 110 * 1024);  // the cost cells: sum |D_i| = k*l
-    ps.lsum2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
+    ps.lsum2 = nw >= 4;
     ps.tpb_ls2 = 32 * (nw + 1);
     ps.smem_ls2 = ps.lsum2 ? ps.lay[KK_LS2].bytes : 0;
     // refinement: two blocks per SM when they fit, else one block with the
     // largest layout under the opt-in limit (long rows, many cells: C4)
     ps.lay[KK_REF2] = ls2_layout((int)kd, nw, 110 * 1024);
-    if (nw < 4 && !getenv("PROCLUS_REF_SMALL")) ps.lay[KK_REF2] = ls2_layout((int)kd, nw, 220 * 1024);
-    ps.ref2 = nw >= 4 && !getenv("PROCLUS_OLD_LSUM");
+    if (nw < 4) ps.lay[KK_REF2] = ls2_layout((int)kd, nw, 220 * 1024);
+    ps.ref2 = nw >= 4;
     ps.tpb_ref2 = 32 * (nw + 1);
     ps.smem_ref2 = ps.ref2 ? ps.lay[KK_REF2].bytes : 0;
   }
@@ -3909,11 +4029,11 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.lab = b.take((size_t)stages * P);
     L.tab = b.take(sizeof(CItem) * kd);
     L.nD = b.take(4 * KMAX);
-    L.acc = b.take(8 * (size_t)nw1 * k * 32);
+    L.acc = b.take(8 * (size_t)L.nw * k * 32);
     finish(L, b, ps.tl);
     ps.lay[KK_COST1] = L;
-    ps.cost1 = L.bytes <= 200 * 1024 && !getenv("PROCLUS_OLD_COST");
-    ps.tpb_cost1 = 32 * (nw1 + 1);
+    ps.cost1 = L.bytes <= 200 * 1024;
+    ps.tpb_cost1 = 32 * (L.nw + 1);
     ps.smem_cost1 = ps.cost1 ? L.bytes : 0;
   }
   ps.smem_loc = ps.lay[KK_LOC].bytes;
@@ -3950,7 +4070,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
                        : d <= 32 ? (const void*)k_locality<32>
                                  : (const void*)k_locality<0>;
   ps.grid_loc = grid_of(loc_fn, ps.smem_loc, ps.tpb_loc);
-  ps.grid_asg = grid_of(ppt2 == 2 ? (const void*)k_assign<2> : (const void*)k_assign<1>,
+  ps.grid_asg = grid_of(ppt2 == 2 ? (const void*)k_assign<2> : (const void*)k_assign_w,
                         ps.smem_asg, ps.tpb_asg);
   ps.grid_lsum = grid_of((const void*)k_labelsum<0>, ps.smem_cost, ps.tpb_lsum);
   ps.grid_fin = grid_of(ppt2 == 2 ? (const void*)k_final<2> : (const void*)k_final<1>,
@@ -3969,7 +4089,7 @@ cudaError_t configure_kernels(const PassShape& ps) {
                        (const void*)k_locality<0>,  (const void*)k_assign<2>,
                        (const void*)k_labelsum<0>,  (const void*)k_labelsum<1>,
                        (const void*)k_final<2>,     (const void*)k_prepare,
-                       (const void*)k_tail,         (const void*)k_assign<1>,
+                       (const void*)k_tail,         (const void*)k_assign_w,
                        (const void*)k_final<1>};
   const size_t sm[] = {ps.smem_loc,  ps.smem_loc, ps.smem_loc,   ps.smem_asg, ps.smem_cost,
                        ps.smem_ref,  ps.smem_fin, (size_t)ps.tail_smem, (size_t)ps.tail_smem,
@@ -4005,16 +4125,10 @@ void launch_locality(const RunParams& p, const PassShape& ps, cudaStream_t s) {
     k_locality<0><<<ps.grid_loc, ps.tpb_loc, ps.smem_loc, s>>>(p);
 }
 void launch_assign(const RunParams& p, const PassShape& ps, cudaStream_t s) {
-  if (ps.ppt2 == 2) {
+  if (ps.ppt2 == 2)
     k_assign<2><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
-  } else if (ps.P_asg == p.P) {
-    k_assign<1><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
-  } else {  // chunks of P_asg points (same 32-point sub-chunks, same sums)
-    RunParams q = p;
-    q.P = ps.P_asg;
-    q.nchunks = (p.n + q.P - 1) / q.P;
-    k_assign<1><<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(q);
-  }
+  else
+    k_assign_w<<<ps.grid_asg, ps.tpb_asg, ps.smem_asg, s>>>(p);
 }
 void launch_cost(const RunParams& p, const PassShape& ps, cudaStream_t s) {
   if (ps.cost1)

@@ -29,6 +29,7 @@ struct PassShape {
   TailLayout tl;
   int tail_smem;
   int split_tails;       // 1: the single-block tails run as kernels of their own (k d > 512)
+  int asg_w;             // 1: long rows, k_assign_w (ASW_NW warps share a chunk)
 };
 
 // N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value;
