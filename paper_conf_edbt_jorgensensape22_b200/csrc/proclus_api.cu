@@ -680,6 +680,7 @@ static proclus_status init_phase(proclus_handle* h, int k_sm, int A, int B, uint
   CK(h->used.ensure((size_t)nM));
   CK(cudaMemsetAsync(h->Hq.p, 0, sizeof(long long) * nM * d, h->stream));
   CK(cudaMemsetAsync(h->nL.p, 0, sizeof(long long) * nM, h->stream));
+  CK(cudaMemsetAsync(h->dprev.p, 0, sizeof(double) * nM, h->stream));  // read only if used
   CK(cudaMemsetAsync(h->found.p, 0, nM, h->stream));
   CK(cudaMemsetAsync(h->used.p, 0, nM, h->stream));
   return PROCLUS_OK;
@@ -775,6 +776,8 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   CK(h->Z.ensure((size_t)KMAX * d));
   CK(h->mu.ensure((size_t)KMAX * d));
   CK(h->dlist.ensure((size_t)KMAX * d));
+  // the rows' tails beyond |D_i| are copied by the passes but never used
+  CK(cudaMemsetAsync(h->dlist.p, 0, sizeof(int) * KMAX * d, h->stream));
   CK(h->dmask.ensure((size_t)KMAX * d));
   CK(h->accg.ensure((size_t)NCOPY * KMAX * d));
   CK(h->cntg.ensure((size_t)NCOPY * KMAX));

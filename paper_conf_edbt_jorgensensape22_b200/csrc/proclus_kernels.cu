@@ -3551,8 +3551,9 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
   const int P = p.P, d = p.d, k = p.k;
   const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const Pipe R = pipe_of(L, smraw, d);
-  CItem* tab = SMP(CItem, tab);
+  CItem* tab = SMP(CItem, tab);            // [k*l]: cluster c's items from off_s[c]
   int* nD_s = SMP(int, nD);
+  int* off_s = SMP(int, off);
   long long* acc_s = SMP(long long, acc);  // [nw][k][32] lane-private columns
   const long long nmy = chunks_of_block(p);
   for (int e = threadIdx.x; e < nw * k * 32; e += blockDim.x) acc_s[e] = 0;
@@ -3562,10 +3563,21 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
   const unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
   for (int i = threadIdx.x; i < k; i += blockDim.x) nD_s[i] = st->nD[i];
   __syncthreads();
+  if (k * d > 512) {  // compact item table (sum |D_i| = k l entries): frees shared memory
+    if (threadIdx.x == 0) {
+      int o = 0;
+      for (int i = 0; i < k; ++i) {
+        off_s[i] = o;
+        o += nD_s[i];
+      }
+    }
+  } else {
+    for (int i = threadIdx.x; i < k; i += blockDim.x) off_s[i] = i * d;
+  }
   const double sc = scalbn(1.0, cost_qexp(p.scale, 1, p.dlist, nD_s, k, d));
   for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
     const int i = e / d, t = e - i * d;
-    if (t < nD_s[i]) tab[e] = CItem{p.dlist[e] * R.ldr * 4, 0, dmul(p.mu[e], sc)};
+    if (t < nD_s[i]) tab[off_s[i] + t] = CItem{p.dlist[e] * R.ldr * 4, 0, dmul(p.mu[e], sc)};
   }
   __syncthreads();
   if (w == nw) {
@@ -3582,7 +3594,7 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
       if (gp < p.n) {
         const int c = R.lab[(size_t)stg * P + q];
         const char* xq = reinterpret_cast<const char*>(R.buf + (size_t)stg * R.rows * R.ldr + q);
-        const CItem* tb = tab + c * d;
+        const CItem* tb = tab + off_s[c];
         const int nd = nD_s[c];
         long long a0 = 0, a1 = 0;
         int t = 0;
@@ -4027,8 +4039,9 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.empty = b.take(8 * SMAX);
     L.buf = b.take((size_t)stages * d * P * 4);
     L.lab = b.take((size_t)stages * P);
-    L.tab = b.take(sizeof(CItem) * kd);
+    L.tab = b.take(sizeof(CItem) * (kd > 512 ? (size_t)k * l : kd));  // compact at large k d
     L.nD = b.take(4 * KMAX);
+    L.off = b.take(4 * (KMAX + 1));
     L.acc = b.take(8 * (size_t)L.nw * k * 32);
     finish(L, b, ps.tl);
     ps.lay[KK_COST1] = L;

@@ -47,11 +47,7 @@ for n, u in rows:
     by[n][0] += 1
     by[n][1] += u
 
-# ---- full capture: per-launch metrics
-raw = subprocess.run(["ncu", "-i", os.path.join(src, "full.ncu-rep"), "--page", "raw", "--csv"],
-                     capture_output=True, text=True).stdout
-rr = list(csv.reader(io.StringIO(raw)))
-hdr, data = rr[0], rr[2:]
+# ---- full captures (every <dir>/full*.ncu-rep): per-launch metrics
 want = {
     "dur_us": "gpu__time_duration.sum",
     "dram_rd_MB": "dram__bytes_read.sum",
@@ -65,30 +61,38 @@ want = {
     "block": "launch__block_size",
     "smem_KB": "launch__shared_mem_per_block_dynamic",
 }
-idx = {k: hdr.index(v) for k, v in want.items() if v in hdr}
-units = rr[1]
 full = []
-for r in data:
-    rec = {"kernel": short(r[hdr.index("Kernel Name")])}
-    for k, i in idx.items():
-        try:
-            val = float(r[i].replace(",", ""))
-        except ValueError:
-            continue
-        u = units[i]
-        if k.startswith("dram_") and k.endswith("MB"):
-            val = val * {"byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3}.get(u, 1.0)
-        if k == "dur_us":
-            val = val * {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}.get(u, 1.0)
-        if k == "inst_M":
-            val = val / 1e6
-        if k == "smem_KB":
-            val = val * {"byte": 1 / 1024, "Kbyte": 1.0, "Mbyte": 1024.0}.get(u, 1.0)
-        rec[k] = round(val, 3)
-    full.append(rec)
+reps = sorted(f for f in os.listdir(src) if f.startswith("full") and f.endswith(".ncu-rep"))
+for rep in reps:
+  raw = subprocess.run(["ncu", "-i", os.path.join(src, rep), "--page", "raw", "--csv"],
+                       capture_output=True, text=True).stdout
+  rr = list(csv.reader(io.StringIO(raw)))
+  hdr, data = rr[0], rr[2:]
+  idx = {k: hdr.index(v) for k, v in want.items() if v in hdr}
+  units = rr[1]
+  for r in data:
+      rec = {"kernel": short(r[hdr.index("Kernel Name")]), "capture": rep}
+      for k, i in idx.items():
+          try:
+              val = float(r[i].replace(",", ""))
+          except ValueError:
+              continue
+          u = units[i]
+          if k.startswith("dram_") and k.endswith("MB"):
+              val = val * {"byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3}.get(u, 1.0)
+          if k == "dur_us":
+              val = val * {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}.get(u, 1.0)
+          if k == "inst_M":
+              val = val / 1e6
+          if k == "smem_KB":
+              val = val * {"byte": 1 / 1024, "Kbyte": 1.0, "Mbyte": 1024.0}.get(u, 1.0)
+          rec[k] = round(val, 3)
+      full.append(rec)
 
 traffic, tcount = {}, {}
 for rec in full:
+    if rec["capture"] != "full.ncu-rep" and rec["capture"] != "full_ac.ncu-rep":
+        continue  # roofline traffic: the C3 workload only
     kname = rec["kernel"]
     base = re.sub(r"<.*", "", kname).replace("k_", "")
     if base in ("lsum2", "labelsum"):
@@ -110,14 +114,16 @@ with open(os.path.join(prof, f"{tag}_ncu_summary.md"), "w") as f:
             "graph with conditional nodes).  Launch list: `ncu --metrics\n"
             "gpu__time_duration.sum --clock-control none` over `bench.py --steps 2\n"
             "--warmup 3` (cold-cache and serialised: compare shares, not absolutes).\n"
-            "Full capture: `ncu --set full --clock-control none` of the C3 pass kernels\n"
-            "(tools/profile_run.py C3 1).\n\n")
+            "Full captures: `ncu --set full --clock-control none` (tools/profile_r02.sh):\n"
+            "full.ncu-rep = C3 k_locality launches 2-5, full_ac.ncu-rep = C3 assign / cost,\n"
+            "full_c4.ncu-rep = C4 (256k x 100) pass kernels and split tails\n"
+            "(tools/profile_run.py C3|C4 1).\n\n")
     f.write("## Share of device time by kernel (launch list)\n\n")
     f.write("| kernel | launches | total us | mean us | share |\n|---|---|---|---|---|\n")
     for n, (c, u) in sorted(by.items(), key=lambda kv: -kv[1][1]):
         f.write(f"| {n} | {c} | {u:.1f} | {u / c:.2f} | {u / tot:.3f} |\n")
     f.write("\n## Full capture, per launch\n\n")
-    cols = ["kernel"] + [k for k in want if any(k in r for r in full)]
+    cols = ["kernel", "capture"] + [k for k in want if any(k in r for r in full)]
     f.write("| " + " | ".join(cols) + " |\n|" + "---|" * len(cols) + "\n")
     for rec in full:
         f.write("| " + " | ".join(str(rec.get(c, "")) for c in cols) + " |\n")
