@@ -26,6 +26,8 @@
 #include <math_constants.h>
 
 #include <algorithm>
+#include <map>
+#include <mutex>
 #include <cstdio>
 #include <cstdlib>
 
@@ -3809,7 +3811,7 @@ static TailLayout tail_layout(int d, int k, int nM) {
   return t;
 }
 
-static bool g_split_tails = false;  // set by pass_shape before the layouts are built
+static thread_local bool g_split_tails = false;  // set by pass_shape (per thread) before the layouts are built
 static void finish(SmemLayout& L, LB& b, const TailLayout& tl) {
   L.tail = L.buf;
   size_t end = b.off;
@@ -4096,8 +4098,27 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   return ps;
 }
 
+// The dynamic shared-memory opt-in is a process-wide attribute of a kernel
+// (per device).  Handles of different shapes may run concurrently from
+// different threads, so the attribute only ever grows: each (device, kernel)
+// is raised to the largest size any handle has needed, under a mutex.
+static std::mutex g_attr_mu;
+static std::map<std::pair<int, const void*>, int> g_attr_max;
+
+static cudaError_t raise_smem(int dev, const void* fn, size_t bytes) {
+  const int want = (int)bytes;
+  auto& cur = g_attr_max[{dev, fn}];
+  if (want <= cur) return cudaSuccess;
+  const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, want);
+  if (e == cudaSuccess) cur = want;
+  return e;
+}
+
 cudaError_t configure_kernels(const PassShape& ps) {
-  cudaError_t e;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(g_attr_mu);
   const void* fns[] = {(const void*)k_locality<16>, (const void*)k_locality<32>,
                        (const void*)k_locality<0>,  (const void*)k_assign<2>,
                        (const void*)k_labelsum<0>,  (const void*)k_labelsum<1>,
@@ -4107,25 +4128,14 @@ cudaError_t configure_kernels(const PassShape& ps) {
   const size_t sm[] = {ps.smem_loc,  ps.smem_loc, ps.smem_loc,   ps.smem_asg, ps.smem_cost,
                        ps.smem_ref,  ps.smem_fin, (size_t)ps.tail_smem, (size_t)ps.tail_smem,
                        ps.smem_asg,  ps.smem_fin};
-  for (int i = 0; i < 11; ++i) {
-    e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm[i]);
-    if (e != cudaSuccess) return e;
-  }
-  if (ps.lsum2) {
-    e = cudaFuncSetAttribute((const void*)k_lsum2<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)ps.smem_ls2);
-    if (e != cudaSuccess) return e;
-  }
-  if (ps.ref2) {
-    e = cudaFuncSetAttribute((const void*)k_lsum2<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)ps.smem_ref2);
-    if (e != cudaSuccess) return e;
-  }
-  if (ps.cost1) {
-    e = cudaFuncSetAttribute((const void*)k_cost1, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)ps.smem_cost1);
-    if (e != cudaSuccess) return e;
-  }
+  for (int i = 0; i < 11; ++i)
+    if ((e = raise_smem(dev, fns[i], sm[i])) != cudaSuccess) return e;
+  if (ps.lsum2 && (e = raise_smem(dev, (const void*)k_lsum2<0>, ps.smem_ls2)) != cudaSuccess)
+    return e;
+  if (ps.ref2 && (e = raise_smem(dev, (const void*)k_lsum2<1>, ps.smem_ref2)) != cudaSuccess)
+    return e;
+  if (ps.cost1 && (e = raise_smem(dev, (const void*)k_cost1, ps.smem_cost1)) != cudaSuccess)
+    return e;
   return cudaSuccess;
 }
 

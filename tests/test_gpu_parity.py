@@ -456,3 +456,45 @@ def test_async_load_rejects_nonfinite_at_run(pk, orc):
         h.load(d1)
         g = h.run(5, 3, seed=1)
     assert_parity(g, orc.proclus(d1, 5, 3, seed=1), what="after a rejected load")
+
+
+@pytest.mark.parametrize("case", ["C1-1", "C1-2", "C2-1"])
+def test_tail_kernels_in_graph(pk, orc, monkeypatch, case):
+    """PROCLUS_TAIL_KERNELS=1: the single-block tails as 1024-thread kernels
+    of their own inside the graph (the default only for k d > 512) give the
+    same clustering at small k d."""
+    monkeypatch.setenv("PROCLUS_TAIL_KERNELS", "1")
+    name, seed = case.split("-")
+    data, cfg = synth.config_data(name, seed=int(seed))
+    g, gt, o, ot = run_both(pk, orc, data, cfg["k"], cfg["l"], seed=int(seed))
+    assert_parity(g, o, gt, ot, what=f"tail kernels {case}")
+
+
+def test_concurrent_handles_of_different_shapes(pk, orc):
+    """Two handles with different shared-memory needs (d = 15 and d = 100)
+    run from two host threads at once: the kernels' dynamic shared-memory
+    opt-in only grows, so neither launch fails."""
+    import threading
+
+    a = synth.generate(4000, 15, 5, 3, seed=61)
+    b = synth.generate(3000, 100, 10, 10, seed=62)
+    out, err = {}, []
+
+    def work(name, data, k, l):
+        try:
+            with pk.Proclus(data) as h:
+                for s in range(3):
+                    out[(name, s)] = h.run(k, l, A=20, B=5, seed=s + 1)
+        except Exception as e:  # noqa: BLE001
+            err.append(e)
+
+    ts = [threading.Thread(target=work, args=("a", a, 5, 3)),
+          threading.Thread(target=work, args=("b", b, 10, 10))]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not err, err
+    for s in range(3):
+        assert_parity(out[("a", s)], orc.proclus(a, 5, 3, A=20, B=5, seed=s + 1), what="a")
+        assert_parity(out[("b", s)], orc.proclus(b, 10, 10, A=20, B=5, seed=s + 1), what="b")
