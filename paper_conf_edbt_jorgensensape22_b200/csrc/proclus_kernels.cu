@@ -1420,6 +1420,22 @@ __device__ void state_store(const RunParams& p, const DevState* S) {
   for (int i = threadIdx.x; i < STATE_WORDS; i += blockDim.x) dst[i] = src[i];
 }
 
+// Position of the (r+1)-th set bit of w (r 0-based, r < popc(w)): a binary
+// search on population counts (the __fns intrinsic is a long sequence).
+__device__ __forceinline__ int nth_set_bit(unsigned w, int r) {
+  int base = 0;
+#pragma unroll
+  for (int sh = 16; sh >= 1; sh >>= 1) {
+    const unsigned low = w & ((1u << sh) - 1u);
+    const int c = __popc(low);
+    const bool up = r >= c;
+    r = up ? r - c : r;
+    w = up ? (w >> sh) : low;
+    base += up ? sh : 0;
+  }
+  return base;
+}
+
 // Warp argmin of (key, j) over keys[0..d) skipping j == excl: smallest key,
 // then smaller j.  Every lane returns the winning j.
 __device__ __forceinline__ int warp_argmin_row(const unsigned long long* keys, int d, int excl) {
@@ -1495,29 +1511,37 @@ __device__ void zscore_select_s(const RunParams& p, TailMem& T, int tq = -1) {
   if (d <= 64) {
     // two smallest per row by (key, j), one thread per row: a sequential
     // scan of d shared keys beats two warp reductions per row here
-    if (tid < k) {
-      const unsigned long long* kr = key + tid * d;
-      unsigned long long b1 = ~0ull, b2 = ~0ull;
-      int j1 = 0, j2 = 1;
-      for (int j = 0; j < d; ++j) {  // ascending j: strict < keeps the smaller j on ties
-        const unsigned long long v = kr[j];
-        if (v < b1) {
-          b2 = b1;
-          j2 = j1;
-          b1 = v;
-          j1 = j;
-        } else if (v < b2) {
-          b2 = v;
-          j2 = j;
-        }
+    // two smallest per row by (key, j): every cell counts the cells of its
+    // row that precede it (d <= 64 compares, all cells in parallel)
+    bool top2 = false;
+    const int c = tid;
+    if (c < kd) {
+      const int i = c / d, j = c - i * d;
+      const unsigned long long* kr = key + i * d;
+      const unsigned long long kc = kr[j];
+      int r = 0;
+      for (int o = 0; o < d; ++o) {
+        const unsigned long long v = kr[o];
+        r += (v < kc) | ((v == kc) & (o < j));
       }
-      dm[tid * d + j1] = 1;
-      dm[tid * d + j2] = 1;
-      if (R > 0) {  // taken cells never rank before a free one
-        key[tid * d + j1] = ~0ull;
-        key[tid * d + j2] = ~0ull;
-      }
+      top2 = r < 2;
+      if (top2) dm[c] = 1;
     }
+    for (int e = tid + bd; e < kd; e += bd) {  // k d > blockDim: the rest
+      const int i = e / d, j = e - i * d;
+      const unsigned long long* kr = key + i * d;
+      const unsigned long long kc = kr[j];
+      int r = 0;
+      for (int o = 0; o < d; ++o) {
+        const unsigned long long v = kr[o];
+        r += (v < kc) | ((v == kc) & (o < j));
+      }
+      if (r < 2) dm[e] = 1;
+    }
+    __syncthreads();  // every row's ranks were taken on the original keys
+    if (R > 0)        // taken cells never rank before a free one
+      for (int e = tid; e < kd; e += bd)
+        if (dm[e]) key[e] = ~0ull;
   } else {
     for (int i = w; i < k; i += nw) {  // two smallest per row, ties -> smaller j
       const int j1 = warp_argmin_row(key + i * d, d, -1);
@@ -2031,7 +2055,7 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
           const int src = __ffs(hit) - 1;
           const int before = __shfl_sync(full, x - c, src);
           const unsigned sw = __shfl_sync(full, wv, src);
-          const int bit = __fns(sw, 0, r - before + 1);
+          const int bit = nth_set_bit(sw, r - before);
           pos = 32 * (w0 + src) + bit;
         } else {
           r -= __shfl_sync(full, x, 31);
