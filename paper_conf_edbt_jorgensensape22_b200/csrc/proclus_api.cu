@@ -839,6 +839,7 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
   s.rng = it;
   for (int i = 0; i < KMAX; ++i) s.cown[i] = -1;
   s.cost_best = INFINITY;
+  s.dbg_t[0] = ~0ull;  // min-reduced entry time of the profiled locality launch
   s.cur_buf = 0;
   s.best_buf = 1;
   launch_put(h->st.p, &s, sizeof(DevState), h->stream);
@@ -1023,6 +1024,9 @@ static proclus_status run_setting(proclus_handle* h, int k, int l, double minDev
       fprintf(stderr, "tail_cycles");
       for (int t = 0; t < 24; ++t) fprintf(stderr, " %llu", h->h_st->dbg_cyc[t]);
       fprintf(stderr, "\n");
+      fprintf(stderr, "loc_phase_ns launches %llu prologue %llu chunks %llu flush %llu tail_start %llu\n",
+              h->h_st->dbg_ts[0], h->h_st->dbg_ts[1], h->h_st->dbg_ts[2], h->h_st->dbg_ts[3],
+              h->h_st->dbg_ts[4]);
     }
   }
   return PROCLUS_OK;

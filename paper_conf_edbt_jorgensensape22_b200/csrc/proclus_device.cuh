@@ -51,6 +51,8 @@ struct DevState {
   long long fallback[4];        // exact fp64 re-decisions (loc, asg, fin, -)
   unsigned long long tail_ns[4];  // %globaltimer time in the single-block tails
   unsigned long long dbg_cyc[24];  // per-phase SM cycles of the tails (PROCLUS_TAIL_PROFILE builds)
+  unsigned long long dbg_t[8];     // k_locality phase times of the current launch (profile builds)
+  unsigned long long dbg_ts[8];    // their sums over the run, ns after the first block's entry
 };
 
 struct TraceBufs {

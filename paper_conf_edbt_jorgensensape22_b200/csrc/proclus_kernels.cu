@@ -1064,22 +1064,24 @@ __device__ __forceinline__ void pipe_release(const Pipe& R, int stg) {
 }
 
 // The last block to arrive (ticket) returns true; it then sees every other
-// block's atomics (threadfence before the ticket, ld.cg reads after).
+// block's atomics (acquire-release ticket, ld.cg reads after).
+// One acquire-release atomic at gpu scope instead of two sequentially
+// consistent fences: the barrier orders the block's flush atomics before
+// thread 0's release (cumulativity), and the last block's acquire plus the
+// barrier order its later L2 (ld.cg) reads after every other block's release.
 __device__ bool last_block(unsigned int* ticket) {
   __shared__ int is_last;
-  __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) {
-    unsigned t = atomicAdd(ticket, 1u);
+    unsigned t;
+    asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(t) : "l"(ticket) : "memory");
     is_last = (t == gridDim.x - 1);
+    if (is_last) *ticket = 0u;
   }
   __syncthreads();
-  if (is_last) {
-    __threadfence();
-    if (threadIdx.x == 0) *ticket = 0u;
-  }
   return is_last;
 }
+
 
 // Combine the per-warp accumulators (exact int64) and add them to one of the
 // NCOPY global copies with one atomic per non-zero cell.  Whole block.
@@ -2506,13 +2508,27 @@ template <int DR>
 #endif
 __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
   DevState* st = p.st;
-  if (st->done) return;
+#ifdef PROCLUS_TAIL_PROFILE
+  if (threadIdx.x == 0) atomicMin(&st->dbg_t[0], gtimer());
+#define LOC_T(idx) \
+  do {             \
+    if (threadIdx.x == 0) atomicMax(&st->dbg_t[idx], gtimer()); \
+  } while (0)
+#else
+#define LOC_T(idx) do {} while (0)
+#endif
   extern __shared__ __align__(16) unsigned char smraw[];
   const SmemLayout& L = p.lay[KK_LOC];
 #define LAYK KK_LOC
   const int d = p.d, k = p.k;
   const int nw = L.nw, w = threadIdx.x >> 5;
-  const int na = st->n_act;
+  // one round trip for the control words: stop flag, |active|, every slot of
+  // the active list (whatever |active| is), 2^e_j
+  __shared__ int ctl_s[2];
+  if (threadIdx.x == 0) {
+    ctl_s[0] = st->done;
+    ctl_s[1] = st->n_act;
+  }
   const int ncap = k * d;
   const Pipe R = pipe_of(L, smraw, DR == 16 && d + k < 16 ? 16 : d + k);
   float* med_s = SMP(float, med);
@@ -2524,40 +2540,57 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
   ExtraRows* ex = SMP(ExtraRows, ex);
   Thr* thr_s = SMP(Thr, thr);
   double* medd_s = DR == 16 ? SMP(double, ctr) : nullptr;          // [na][16] fp64 medoid rows
+#ifdef LOC_EMPTY
+  const long long nmy = 0;  // timing experiment only: prologue, epilogue and tail
+#else
   const long long nmy = chunks_of_block(p);
+#endif
   const double G = (double)(d + 8) * 5.9604644775390625e-08;  // (d+8) 2^-24
 
-  for (int a = threadIdx.x; a < na; a += blockDim.x) {
-    act_s[a] = st->act[a];
-    thr_s[a] = make_thr(st->act[a].lo, st->act[a].hi, G);
+  for (int a = threadIdx.x; a < KMAX; a += blockDim.x) {
+    const ActSlot A = st->act[a];  // slots >= |active| are stale and unused
+    act_s[a] = A;
+    thr_s[a] = make_thr(A.lo, A.hi, G);
   }
   for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
   for (int e = threadIdx.x; e < (DR == 16 ? nw : 1) * ncap; e += blockDim.x) acc_s[e] = 0;
   for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
   pipe_init(p, R, nw);
   __syncthreads();
-  if (threadIdx.x < 32) {  // rows of the cached slots (warp ballot scan)
-    const int a = threadIdx.x;
+  if (ctl_s[0]) return;
+  const int na = ctl_s[1];
+  if (threadIdx.x < 32 || w == nw) {  // rows of the cached slots (warp ballot scan);
+    // the producer warp derives the same list for its own TMA, so that the
+    // ring starts filling while the consumers load the medoid rows
+    const int a = threadIdx.x & 31;
     const bool cached = a < na && !act_s[a].compute;
     const unsigned b = __ballot_sync(0xffffffffu, cached);
     const int r = __popc(b & ((1u << a) - 1u));
-    if (a < na) row_s[a] = cached ? (d + r) * R.ldr : -1;
-    if (cached) ex->src[r] = p.dist + (size_t)act_s[a].key * p.n_pad;
-    if (a == 0) ex->n = __popc(b);
+    if (w == 0) {
+      if (a < na) row_s[a] = cached ? (d + r) * R.ldr : -1;
+    } else {
+      if (cached) ex->src[r] = p.dist + (size_t)act_s[a].key * p.n_pad;
+      if (a == 0) ex->n = __popc(b);
+      __syncwarp();
+    }
   }
   // medoid rows at stride MS (zero padded to DR for float4 loads)
   constexpr int MSD = DR > 0 ? DR : 0;
   const int MS = MSD > 0 ? MSD : d;
-  for (int e = threadIdx.x; e < na * MS; e += blockDim.x) {
-    const int a = e / MS, j = e - a * MS;
-    const float m = j < d ? p.mrows[(long long)act_s[a].mpos * d + j] : 0.f;
-    med_s[e] = m;
-    if (DR == 16) medd_s[e] = (double)m;
+  if (w < nw) {
+    for (int e = threadIdx.x; e < na * MS; e += nw * 32) {
+      const int a = e / MS, j = e - a * MS;
+      const float m = j < d ? p.mrows[(long long)act_s[a].mpos * d + j] : 0.f;
+      med_s[e] = m;
+      if (DR == 16) medd_s[e] = (double)m;
+    }
+    named_bar_sync(2, nw * 32);  // consumers only: the producer is already streaming
   }
-  __syncthreads();
+  LOC_T(1);  // prologue done
   long long nfb = 0;
-  int ncomp = 0;  // active slots whose Dist row is computed in this pass
-  for (int a = 0; a < na; ++a) ncomp += row_s[a] < 0;
+  int ncomp = 0;  // active slots whose Dist row is computed in this pass (consumers)
+  if (w < nw)
+    for (int a = 0; a < na; ++a) ncomp += row_s[a] < 0;
   if (na > 0) {
     if (w == nw) {
       pipe_produce(p, R, nmy, nullptr, ex);
@@ -2581,12 +2614,28 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
                         cnt_s, scale_s, nfb);
     }
   }
+  LOC_T(2);  // this block's chunks done
   __syncthreads();
   flush_warps(p, acc_s, nw, ncap, na * d, cnt_s, na, DR == 16 ? nw : 1);
   if (nfb) atomicAdd((unsigned long long*)&st->fallback[0], (unsigned long long)nfb);
+  LOC_T(3);  // flushed
   if (!p.fuse_tail) return;
   if (!last_block(&st->ticket[0])) return;
+#ifdef PROCLUS_TAIL_PROFILE
+  if (threadIdx.x == 0) {
+    const unsigned long long t0 = __ldcg(&st->dbg_t[0]);
+    st->dbg_ts[1] += __ldcg(&st->dbg_t[1]) - t0;
+    st->dbg_ts[2] += __ldcg(&st->dbg_t[2]) - t0;
+    st->dbg_ts[3] += __ldcg(&st->dbg_t[3]) - t0;
+    st->dbg_ts[4] += gtimer() - t0;  // tail start (after the ticket)
+    st->dbg_ts[0] += 1;
+    st->dbg_t[0] = ~0ull;
+    st->dbg_t[1] = st->dbg_t[2] = st->dbg_t[3] = 0ull;
+  }
+  __syncthreads();  // before the tail's state_load reads these words
+#endif
   RUN_TAIL(tail_locality, 0);
+#undef LOC_T
 #undef LAYK
 }
 
@@ -4132,6 +4181,16 @@ static std::map<std::pair<int, const void*>, int> g_attr_max;
 static cudaError_t raise_smem(int dev, const void* fn, size_t bytes) {
   const int want = (int)bytes;
   auto& cur = g_attr_max[{dev, fn}];
+  if (cur == 0) {
+#ifdef SMEM_CARVEOUT
+    // one L1 / shared-memory split for every pass kernel: no carve-out
+    // reconfiguration between consecutive kernels of an iteration
+    const cudaError_t ec = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                                cudaSharedmemCarveoutMaxShared);
+    if (ec != cudaSuccess) return ec;
+#endif
+    cur = -1;
+  }
   if (want <= cur) return cudaSuccess;
   const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, want);
   if (e == cudaSuccess) cur = want;
