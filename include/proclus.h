@@ -182,7 +182,12 @@ PROCLUS_API proclus_status proclus_create_ex(const float* data, int64_t n, int32
                                  proclus_handle** out);
 
 /* Replace the handle's data with new values of the same shape (host or
- * device pointer per the handle's options).  Drops all cached distances. */
+ * device pointer per the handle's options).  Drops all cached distances.
+ * With world_size 1 the load is asynchronous on the handle's stream (copy,
+ * pack and the fixed-point scales run on the device): the caller may reuse
+ * a host buffer only after the next proclus_run returns, and a non-finite
+ * value makes that proclus_run fail with EINVAL (proclus_create still
+ * validates synchronously).  EINVAL: NULL arguments. */
 PROCLUS_API proclus_status proclus_load(proclus_handle* h, const float* data);
 
 /* Start copying the NEXT dataset `data` (host pointer, row-major n x d fp32

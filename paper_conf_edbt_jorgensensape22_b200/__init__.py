@@ -277,6 +277,7 @@ class Proclus:
         self.h = proclus_create_ex(data, self.n, self.d, o)
         self._k = None
         self._pf = None  # the array of a pending prefetch (kept alive)
+        self._loaded = None  # the array of the last (asynchronous) load
 
     def close(self):
         if getattr(self, "h", None):
@@ -328,6 +329,7 @@ class Proclus:
         data = self._checked_data(data, copy_ok=True)
         proclus_load(self.h, data)
         self._pf = None  # the prefetched buffer is no longer referenced by the library
+        self._loaded = data  # the asynchronous copy may still read it until the next run
 
     def prefetch(self, data):
         """Start the H2D copy of the next dataset (keep `data` unchanged until
@@ -365,6 +367,7 @@ class Proclus:
             itrPat: int = 5, seed: int = 1, labels=None) -> Result:
         r, lab, med, dims = self._result_struct(k, labels)
         proclus_run(self.h, k, l, A, B, minDev, itrPat, seed, r)
+        self._loaded = None
         self._k = k
         return Result(lab, med, dims.astype(bool), float(r.cost), int(r.iterations))
 
