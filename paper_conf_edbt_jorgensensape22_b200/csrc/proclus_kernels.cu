@@ -2241,6 +2241,16 @@ __device__ __forceinline__ long long quant_sum(double s, double sc, int magic) {
 // 1024-aligned shard boundaries.
 constexpr int LOC16_PPT = 1;  // 2 measured slower (fewer warps per SM)
 
+// The exact fp64 band decision of a point whose fp32 distance is within the
+// error bound (rare): out of line, so that its registers do not count
+// against the consumer loop.
+__device__ __noinline__ bool exact_band(const float* __restrict__ x, int LD,
+                                        const float* __restrict__ m, int d, int metric,
+                                        double lo, double hi) {
+  const double dv = full_dist(x, LD, m, d, metric);
+  return (dv > lo) && (dv <= hi);
+}
+
 // Shared memory is addressed through 32-bit offsets from the dynamic
 // shared-memory base (generic 64-bit pointers cost an IMAD + LEA per access).
 // explicit 32-bit shared-window addressing from a base computed once per
@@ -2344,10 +2354,8 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
         bool in = f < t.in_hi && f > t.out_lo;
         if (valid && !in && !(f > t.out_hi || f < t.in_lo)) {
           // within the fp32 error bound: the oracle's fp64 value decides
-          const ActSlot A = act_s[a];
-          const double dv = full_dist(reinterpret_cast<const float*>(smraw) + xq + 32 * u, LD,
-                                      med_s + a * 16, d, METRIC);
-          in = (dv > A.lo) && (dv <= A.hi);
+          in = exact_band(reinterpret_cast<const float*>(smraw) + xq + 32 * u, LD,
+                          med_s + a * 16, d, METRIC, act_s[a].lo, act_s[a].hi);
           ++nfb;
         }
         in = in && valid;
