@@ -2776,178 +2776,6 @@ __device__ __noinline__ void dist_terms_n(const float* __restrict__ xq, const Te
   for (int u = 0; u < PPT; ++u) s[u] = a[u] + b[u];
 }
 
-template <int PPT>
-__global__ void __launch_bounds__(160) k_assign(RunParams p) {
-  DevState* st = p.st;
-  extern __shared__ __align__(16) unsigned char smraw[];
-  const SmemLayout& L = p.lay[KK_ASG];
-#define LAYK KK_ASG
-  const int P = p.P, d = p.d, k = p.k;
-  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int ncap = k * d;
-  // PPT == 1 (long rows, chunk of 2 P): one accumulator copy shared by the
-  // consumer warps (shared-memory atomics) so that 4 of them fit in a block
-  constexpr bool SHACC = PPT == 1;
-  const int nacc = SHACC ? 1 : nw;
-  const Pipe R = pipe_of(L, smraw, d);
-  float* med_s = SMP(float, med);
-  Term* tab_s = SMP(Term, tab);
-  int* dl_s = SMP(int, dl);
-  int* nD_s = SMP(int, nD);
-  int* off_s = SMP(int, off);
-  float* rcp_s = SMP(float, rcp);
-  double* scale_s = SMP(double, scale);
-  Cell* cells = SMP(Cell, cells);
-  unsigned* bal_s = SMP(unsigned, bal);
-  long long* acc_s = SMP(long long, acc);
-  long long* cnt_s = SMP(long long, cnt);
-  const long long nmy = chunks_of_block(p);
-  // independent of the previous pass: accumulators, ring, first data copies
-  for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
-  for (int e = threadIdx.x; e < nacc * ncap; e += blockDim.x) acc_s[e] = 0;
-  for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
-  pipe_init(p, R, nw);
-  __syncthreads();
-  if (st->done) return;
-  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
-  for (int i = threadIdx.x; i < k; i += blockDim.x) {
-    nD_s[i] = st->nD[i];
-    rcp_s[i] = 1.0f / (float)st->nD[i];
-  }
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
-    const int i = e / d;
-    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
-    dl_s[e] = p.dlist[e];
-  }
-  __syncthreads();
-  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
-    const int i = e / d, t = e - i * d;
-    if (t < nD_s[i]) {
-      const int j = dl_s[e];
-      tab_s[e].joff = j * P * 4;
-      tab_s[e].m = med_s[i * d + j];
-      tab_s[e].m2 = med_s[i * d + j];
-    }
-  }
-  const int ncell = build_cells(cells, nD_s, k, d, off_s, dl_s, nullptr);
-  int ndmax = 0;
-  for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
-  const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
-  long long nfb = 0;
-  if (w == nw) {
-    pipe_produce(p, R, nmy, nullptr, nullptr);
-  } else {
-    unsigned* bal = bal_s + w * KMAX * PPT;
-    long long* acc = acc_s + (SHACC ? (size_t)0 : (size_t)w * ncap);
-    const int q0 = w * 32 * PPT;
-    // PPT == 2: a lane owns the adjacent points q0 + 2 lane + u (packed terms)
-    constexpr bool IL = PPT == 2;
-    long long base = (long long)blockIdx.x * P;
-    const long long gstep = (long long)gridDim.x * P;
-    RingPos rp;
-    for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
-      const int stg = rp.stg;
-      mbar_wait(R.full_a + 8u * stg, rp.ph);
-      const float* xs = R.buf + (size_t)stg * R.rows * P;
-      const float* xq = xs + q0 + (IL ? 2 * lane : lane);
-      float best[PPT], second[PPT];
-      int bi[PPT];
-#pragma unroll
-      for (int u = 0; u < PPT; ++u) {
-        best[u] = CUDART_INF_F;
-        second[u] = CUDART_INF_F;
-        bi[u] = 0;
-      }
-      const Term* tb = tab_s;
-      for (int c = 0; c < k; ++c, tb += d) {
-        const int nd = nD_s[c];
-        // fp32 partial sums in any order: the certified bound only needs the
-        // number of terms (DESIGN.md section 5); 4 terms in flight per point
-        float s[PPT];
-        if constexpr (IL) {
-          switch (nd) {
-#define DT(N) \
-  case N:     \
-    dist_terms2<N>(xq, tb, s); \
-    break;
-            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
-            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
-#undef DT
-            default:
-              dist_terms2_n(xq, tb, nd, s);
-          }
-        } else {
-          switch (nd) {
-#define DT(N) \
-  case N:     \
-    dist_terms<PPT, N>(xq, tb, s); \
-    break;
-            DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
-            DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
-#undef DT
-            default:
-              dist_terms_n<PPT>(xq, tb, nd, s);
-          }
-        }
-        const float r = rcp_s[c];
-#pragma unroll
-        for (int u = 0; u < PPT; ++u) {
-          const float qv = s[u] * r;
-          second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);
-          bi[u] = qv < best[u] ? c : bi[u];
-          best[u] = fminf(best[u], qv);
-        }
-      }
-      int lbl[PPT];
-#pragma unroll
-      for (int u = 0; u < PPT; ++u) {
-        const int q = IL ? q0 + 2 * lane + u : q0 + u * 32 + lane;
-        const long long gp = base + q;
-        lbl[u] = -1;
-        if (gp >= p.n) continue;
-        const bool certain = (best[u] >= 1e-30f) && (second[u] < 1e30f) &&
-                             ((double)second[u] * (1.0 - G) > (double)best[u] * (1.0 + G));
-        lbl[u] = bi[u];
-        if (!certain) {
-          lbl[u] = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
-          ++nfb;
-        }
-        lab[gp] = (unsigned char)lbl[u];
-      }
-      {  // one ballot per (cluster, u): lane c keeps cluster c's masks
-        unsigned mine[PPT];
-#pragma unroll
-        for (int u = 0; u < PPT; ++u) mine[u] = 0u;
-        for (int c = 0; c < k; ++c)
-#pragma unroll
-          for (int u = 0; u < PPT; ++u) {
-            const unsigned b = __ballot_sync(0xffffffffu, lbl[u] == c);
-            if (lane == c) mine[u] = b;
-          }
-        if (lane < k) {
-          int cn = 0;
-#pragma unroll
-          for (int u = 0; u < PPT; ++u) {
-            bal[lane * PPT + u] = mine[u];
-            cn += __popc(mine[u]);
-          }
-          cnt_s[w * KMAX + lane] += cn;
-        }
-      }
-      __syncwarp();
-      warp_cells<0, PPT, IL, SHACC>(xs, P, q0, cells, ncell, bal, acc, scale_s);
-      pipe_release(R, stg);
-    }
-  }
-  __syncthreads();
-  flush_warps(p, acc_s, nw, ncap, k * d, cnt_s, k, nacc);
-  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
-  if (!p.fuse_tail) return;
-  if (!last_block(&st->ticket[1])) return;
-  RUN_TAIL(tail_assign, 1);
-#undef LAYK
-}
-
 // --- AssignPoints (Alg 5) + centroid sums for long rows (chunks of P <= 64
 // points): the ASW_NW consumer warps share every chunk instead of owning 32
 // points each (round 1 ran C4 with 4 consumer warps per SM).
@@ -3525,6 +3353,155 @@ __device__ __forceinline__ void pipe_init_k(const SmemLayout& L, const Pipe& R) 
   }
 }
 
+// --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8),
+// chunks of >= 128 points.  A lane owns the adjacent points q0 + 2 lane + u
+// (u = 0, 1) of its warp's 64 columns: certified fp32 argmin over the
+// clusters (packed terms, one switch per cluster on the warp-uniform |D_c|),
+// fp64 fallback near a tie (reading R8), u8 label.  Then the chunk is
+// counting-sorted by the new labels among the consumer threads and the item
+// threads (cell (c, t), residue r, stride R_c ~ |C_c|) add round(x_j 2^e_j)
+// of the members in registers: exact int64 centroid sums, independent of the
+// order, the grid and the GPU count, with no per-cluster ballots or bit walks.
+template <int PPT>
+__global__ void __launch_bounds__(160) k_assign(RunParams p) {
+  static_assert(PPT == 2, "two adjacent points per lane");
+  DevState* st = p.st;
+  extern __shared__ __align__(16) unsigned char smraw[];
+  const SmemLayout& L = p.lay[KK_ASG];
+#define LAYK KK_ASG
+  const int P = p.P, d = p.d, k = p.k;
+  const int nw = L.nw, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int nct = nw * 32;
+  const Pipe R = pipe_of(L, smraw, d);
+  float* med_s = SMP(float, med);
+  Term* tab_s = SMP(Term, tab);
+  int* dl_s = SMP(int, dl);
+  int* nD_s = SMP(int, nD);
+  float* rcp_s = SMP(float, rcp);
+  __shared__ int off_s[KMAX], ndi_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
+  ItemCtx X;
+  X.items = SMP(Item, cells);
+  X.iacc = SMP(long long, acc);
+  X.gix = SMP(int, ctr);
+  X.hist0 = SMP(int, bal);
+  X.list0 = SMP(int, row);
+  X.ccnt = SMP(long long, cnt);
+  X.off_s = off_s;
+  X.nd_s = ndi_s;
+  X.rr_s = rr_s;
+  X.ib_s = ib_s;
+  X.nct = nct;
+  X.nitem = 0;
+  const long long nmy = chunks_of_block(p);
+  pipe_init(p, R, nw);
+  __syncthreads();
+  if (st->done) return;
+  unsigned char* lab = st->cur_buf ? p.lab1 : p.lab0;
+  for (int i = threadIdx.x; i < k; i += blockDim.x) {
+    nD_s[i] = st->nD[i];
+    rcp_s[i] = 1.0f / (float)st->nD[i];
+  }
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d;
+    med_s[e] = p.mrows[(long long)st->mcur[i] * d + (e - i * d)];
+    dl_s[e] = p.dlist[e];
+  }
+  items_build<2>(p, L, X);  // block-wide (barrier inside)
+  __syncthreads();
+  for (int e = threadIdx.x; e < k * d; e += blockDim.x) {
+    const int i = e / d, t = e - i * d;
+    if (t < nD_s[i]) {
+      const int j = dl_s[e];
+      tab_s[e].joff = j * P * 4;
+      tab_s[e].m = med_s[i * d + j];
+      tab_s[e].m2 = med_s[i * d + j];
+    }
+  }
+  __syncthreads();
+  int ndmax = 0;
+  for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
+  const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
+  long long nfb = 0;
+  if (w == nw) {
+    pipe_produce(p, R, nmy, nullptr, nullptr);
+  } else {
+    const int q0 = w * 64, tq = threadIdx.x;
+    long long base = (long long)blockIdx.x * P;
+    const long long gstep = (long long)gridDim.x * P;
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, base += gstep, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      const int hb = (int)(i & 1);
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
+      const float* xs = R.buf + (size_t)stg * R.rows * P;
+      const float* xq = xs + q0 + 2 * lane;
+      float best[2], second[2];
+      int bi[2];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        best[u] = CUDART_INF_F;
+        second[u] = CUDART_INF_F;
+        bi[u] = 0;
+      }
+      const Term* tb = tab_s;
+      for (int c = 0; c < k; ++c, tb += d) {
+        // fp32 partial sums in any order: the certified bound only needs the
+        // number of terms (DESIGN.md section 5); 4 terms in flight per point
+        float s[2];
+        switch (nD_s[c]) {
+#define DT(N) \
+  case N:     \
+    dist_terms2<N>(xq, tb, s); \
+    break;
+          DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+          DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+#undef DT
+          default:
+            dist_terms2_n(xq, tb, nD_s[c], s);
+        }
+        const float r = rcp_s[c];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const float qv = s[u] * r;
+          second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);
+          bi[u] = qv < best[u] ? c : bi[u];
+          best[u] = fminf(best[u], qv);
+        }
+      }
+      int qq[2], cc[2];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int q = q0 + 2 * lane + u;
+        const long long gp = base + q;
+        qq[u] = q;
+        cc[u] = -1;
+        if (gp >= p.n) continue;
+        const bool certain = (best[u] >= 1e-30f) && (second[u] < 1e30f) &&
+                             ((double)second[u] * (1.0 - G) > (double)best[u] * (1.0 + G));
+        int lbl = bi[u];
+        if (!certain) {
+          lbl = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, nullptr, nullptr);
+          ++nfb;
+        }
+        lab[gp] = (unsigned char)lbl;
+        cc[u] = lbl;
+      }
+      sort_chunk_m<2>(qq, cc, nct, k, X.hist0 + hb * KMAX, X.hist0 + (hb ^ 1) * KMAX,
+                      X.hist0 + 2 * KMAX + hb * KMAX, X.list0 + hb * P);
+      items_chunk<2>(X, reinterpret_cast<const char*>(xs), X.hist0 + hb * KMAX,
+                     X.hist0 + 2 * KMAX + hb * KMAX, X.list0 + hb * P, tq, k);
+      pipe_release(R, stg);
+    }
+  }
+  __syncthreads();
+  items_flush<2>(p, X);
+  if (nfb) atomicAdd((unsigned long long*)&st->fallback[1], (unsigned long long)nfb);
+  if (!p.fuse_tail) return;
+  if (!last_block(&st->ticket[1])) return;
+  RUN_TAIL(tail_assign, 1);
+#undef LAYK
+}
+
 // --- EvaluateCluster deviations (Alg 6 l.9-13, eq 9) / refinement X over
 // CBest (Alg 1 l.16-17).  Each chunk is counting-sorted by cluster; every
 // consumer thread owns a fixed set of work items (cell, residue r, stride
@@ -3970,7 +3947,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
   // per-block cluster tables dominate the shared memory at large k d)
   auto asg_layout = [&](int Pa) {
     const int nwa = Pa / (32 * ppt2);
-    const int nacc = ppt2 == 1 ? 1 : nwa;
+    const int imax = 32 * nwa + (int)kd;  // items: sum_i |D_i| R_i <= threads + cells
     SmemLayout L = blank_layout();
     LB b;
     L.nw = nwa;
@@ -3983,13 +3960,13 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.tab = b.take(sizeof(Term) * kd);
     L.dl = b.take(4 * kd);
     L.nD = b.take(4 * KMAX);
-    L.off = b.take(4 * (KMAX + 1));
     L.rcp = b.take(4 * KMAX);
-    L.scale = b.take(8 * (size_t)d);
-    L.cells = b.take(sizeof(Cell) * kd);
-    L.bal = b.take(4 * (size_t)nwa * KMAX * 2);
-    L.acc = b.take(8 * (size_t)nacc * kd);
-    L.cnt = b.take(8 * (size_t)nwa * KMAX);
+    L.cells = b.take(sizeof(Item) * (size_t)imax);  // centroid items
+    L.acc = b.take(8 * (size_t)imax);               // their int64 sums
+    L.ctr = b.take(4 * kd);                         // cell -> accumulator index
+    L.bal = b.take(4 * 4 * KMAX);                   // histograms + bases (double buffer)
+    L.row = b.take(4 * 2 * (size_t)Pa);             // sorted chunk points (double buffer)
+    L.cnt = b.take(8 * KMAX);                       // |C_i| of the block
     finish(L, b, ps.tl);
     return L;
   };
