@@ -3362,6 +3362,16 @@ __device__ __forceinline__ void pipe_init_k(const SmemLayout& L, const Pipe& R) 
 // threads (cell (c, t), residue r, stride R_c ~ |C_c|) add round(x_j 2^e_j)
 // of the members in registers: exact int64 centroid sums, independent of the
 // order, the grid and the GPU count, with no per-cluster ballots or bit walks.
+#define ASG_UPD(c, s)                                                       \
+  do {                                                                      \
+    const float r_ = rcp_s[c];                                              \
+    _Pragma("unroll") for (int u = 0; u < 2; ++u) {                         \
+      const float qv = (s)[u] * r_;                                         \
+      second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);            \
+      bi[u] = qv < best[u] ? (c) : bi[u];                                   \
+      best[u] = fminf(best[u], qv);                                         \
+    }                                                                       \
+  } while (0)
 template <int PPT>
 __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   static_assert(PPT == 2, "two adjacent points per lane");
@@ -3379,6 +3389,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
   int* nD_s = SMP(int, nD);
   float* rcp_s = SMP(float, rcp);
   __shared__ int off_s[KMAX], ndi_s[KMAX], rr_s[KMAX], ib_s[KMAX + 1];
+  __shared__ int ord_s[KMAX], gst_s[KMAX + 1], gnd_s[KMAX], ngrp_s;
   ItemCtx X;
   X.items = SMP(Item, cells);
   X.iacc = SMP(long long, acc);
@@ -3418,6 +3429,33 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     }
   }
   __syncthreads();
+  if (threadIdx.x < 32) {  // clusters ordered by (|D_c|, c), groups of equal |D_c|
+    const int c = lane;
+    const int nd = c < k ? nD_s[c] : 1 << 30;
+    int rank = 0;
+    for (int o = 0; o < k; ++o) {
+      const int no = nD_s[o];
+      rank += (no < nd) | ((no == nd) & (o < c));
+    }
+    if (c < k) ord_s[rank] = c;
+    __syncwarp();
+    const int r = lane;
+    const int ndr = r < k ? nD_s[ord_s[r]] : -1;
+    const int ndp = __shfl_up_sync(0xffffffffu, ndr, 1);
+    const bool head = r < k && (r == 0 || ndp != ndr);
+    const unsigned hb = __ballot_sync(0xffffffffu, head);
+    if (head) {
+      const int g = __popc(hb & ((1u << lane) - 1u));
+      gst_s[g] = r;
+      gnd_s[g] = ndr;
+    }
+    if (lane == 0) {
+      ngrp_s = __popc(hb);
+      gst_s[__popc(hb)] = k;
+    }
+  }
+  __syncthreads();
+  const int ngrp = ngrp_s;
   int ndmax = 0;
   for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
   const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
@@ -3443,29 +3481,30 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
         second[u] = CUDART_INF_F;
         bi[u] = 0;
       }
-      const Term* tb = tab_s;
-      for (int c = 0; c < k; ++c, tb += d) {
-        // fp32 partial sums in any order: the certified bound only needs the
-        // number of terms; 4 terms in flight per point
-        float s[2];
-        switch (nD_s[c]) {
-#define DT(N) \
-  case N:     \
-    dist_terms2<N>(xq, tb, s); \
+      // clusters grouped by |D_c| (one switch per group; the argmin does not
+      // depend on the visiting order: an exact fp32 tie is never certified)
+      for (int g = 0; g < ngrp; ++g) {
+        const int r0 = gst_s[g], r1 = gst_s[g + 1];
+        switch (gnd_s[g]) {
+#define DT(N)                                              \
+  case N:                                                  \
+    for (int r = r0; r < r1; ++r) {                        \
+      const int c = ord_s[r];                              \
+      float s[2];                                          \
+      dist_terms2<N>(xq, tab_s + c * d, s);                \
+      ASG_UPD(c, s);                                       \
+    }                                                      \
     break;
           DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
           DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
 #undef DT
           default:
-            dist_terms2_n(xq, tb, nD_s[c], s);
-        }
-        const float r = rcp_s[c];
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-          const float qv = s[u] * r;
-          second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);
-          bi[u] = qv < best[u] ? c : bi[u];
-          best[u] = fminf(best[u], qv);
+            for (int r = r0; r < r1; ++r) {
+              const int c = ord_s[r];
+              float s[2];
+              dist_terms2_n(xq, tab_s + c * d, gnd_s[g], s);
+              ASG_UPD(c, s);
+            }
         }
       }
       int qq[2], cc[2];
