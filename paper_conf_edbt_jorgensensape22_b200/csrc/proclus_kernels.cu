@@ -992,7 +992,9 @@ __device__ __forceinline__ unsigned long long gtimer() {
 
 struct ExtraRows {
   int n;
+  int row0;                // ring row of the first extra row
   const float* src[KMAX];  // global row bases (indexed by point)
+  float* drow[KMAX];       // k_locality: Dist row of active slot a (new rows are stored there)
 };
 
 struct Pipe {
@@ -1034,7 +1036,8 @@ __device__ void pipe_produce(const RunParams& p, const Pipe& R, long long nmy,
     float* dst = R.buf + (size_t)stg * R.rows * R.ldr;
     for (int j = lane; j < p.d + nex; j += 32) {
       const float* src = j < p.d ? p.xs + (size_t)j * p.n_pad + base : ex->src[j - p.d] + base;
-      bulk_g2s(dst + (size_t)j * R.ldr, src, row, R.full_a + 8u * stg);
+      const int jr = j < p.d ? j : ex->row0 + (j - p.d);
+      bulk_g2s(dst + (size_t)jr * R.ldr, src, row, R.full_a + 8u * stg);
     }
     if (labsrc && lane == 0)
       bulk_g2s(R.lab + (size_t)stg * p.P, labsrc + base, (unsigned)p.P, R.full_a + 8u * stg);
@@ -1923,8 +1926,35 @@ __device__ void tail_cost(const RunParams& p, TailMem& T) {
   }
   for (int j = tid; j < d; j += bd) T.isc[j] = p.iscale[j];
   if (T.mrow) {
-    for (int e = tid; e < nM * d; e += bd) T.mrow[e] = p.mrows[e];
-    for (int m = tid; m < nM; m += bd) {
+    // every load of a thread is issued before its first shared-memory store
+    // (the compiler cannot reorder them across a possibly aliasing store)
+    constexpr int MR = 8;
+    const int nmd = nM * d;
+    float mv[MR];
+#pragma unroll
+    for (int q = 0; q < MR; ++q) {
+      const int e = tid + q * bd;
+      mv[q] = e < nmd ? __ldcg(p.mrows + e) : 0.f;
+    }
+    unsigned char fv = 0, uv = 0;
+    double pv = 0.0;
+    if (tid < nM) {
+      fv = __ldcg(p.found + tid);
+      uv = __ldcg(p.used + tid);
+      pv = __ldcg(p.dprev + tid);
+    }
+#pragma unroll
+    for (int q = 0; q < MR; ++q) {
+      const int e = tid + q * bd;
+      if (e < nmd) T.mrow[e] = mv[q];
+    }
+    for (int e = tid + MR * bd; e < nmd; e += bd) T.mrow[e] = p.mrows[e];
+    if (tid < nM) {
+      T.fall[tid] = fv;
+      T.uall[tid] = uv;
+      T.pall[tid] = pv;
+    }
+    for (int m = tid + bd; m < nM; m += bd) {
       T.fall[m] = p.found[m];
       T.uall[m] = p.used[m];
       T.pall[m] = p.dprev[m];
@@ -2191,7 +2221,7 @@ __device__ int build_cells(Cell* cells, const int* nD_s, int k, int d, int* off_
 // fp32 certified thresholds of one band (lo, hi]: a fp32 value f with
 // |f - v| <= G v decides v <= T when f < T(1-G) (then "<=") or f > T(1+G)
 // (then ">"); the bounds are rounded outwards to fp32 once per launch.
-struct Thr {
+struct __align__(16) Thr {
   float in_hi, out_hi;  // f < in_hi: v <= hi;  f > out_hi: v > hi
   float in_lo, out_lo;  // f > out_lo: v > lo;  f < in_lo: v <= lo
 };
@@ -2300,7 +2330,8 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
                                               const double* __restrict__ medd_s,
                                               const int* __restrict__ row_s,
                                               const Thr* __restrict__ thr_s,
-                                              const ActSlot* __restrict__ act_s, int lst_b,
+                                              const ActSlot* __restrict__ act_s,
+                                              const ExtraRows* __restrict__ ex, int lst_b,
                                               long long* __restrict__ acc,
                                               long long* __restrict__ cnt,
                                               const double* __restrict__ scale_s, long long& nfb) {
@@ -2315,8 +2346,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
   const double sc = scale_s[j < d ? j : 0];
   const int magic = *p.qflag;
   const int variant = p.variant;
-  const long long n = p.n, n_pad = p.n_pad;
-  float* const dist = p.dist;
+  const long long n = p.n;
   long long gp = (long long)blockIdx.x * P + c0 + lane;
   const long long gstep = (long long)gridDim.x * P;
   RingPos rp;
@@ -2329,10 +2359,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
     float x[16];
     if (ncomp > 0) {  // coordinates in registers when a Dist row is computed; rows >= d are 0
 #pragma unroll
-      for (int jj = 0; jj < 16; ++jj) {
-        const float v = SMF(xq + jj * LD);
-        x[jj] = jj < d ? v : 0.f;
-      }
+      for (int jj = 0; jj < 16; ++jj) x[jj] = SMF(xq + jj * LD);
     }
 #ifdef LOC_NOP
     if (na > 0) { pipe_release(R, stg); continue; }  // timing experiment only
@@ -2347,7 +2374,7 @@ __device__ __forceinline__ void loc16_consume(const RunParams& p, const Pipe& R,
         float f;
         if (rs < 0) {  // a new Dist row
           f = loc16_dist<METRIC>(x, med_s + a * 16);
-          if (variant != 1 && valid) dist[(long long)act_s[a].key * n_pad + gp + 32 * u] = f;
+          if (variant != 1 && valid) ex->drow[a][gp + 32 * u] = f;
         } else {
           f = SMF(xq + rs + 32 * u);
         }
@@ -2538,7 +2565,10 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
     ctl_s[1] = st->n_act;
   }
   const int ncap = k * d;
-  const Pipe R = pipe_of(L, smraw, DR == 16 && d + k < 16 ? 16 : d + k);
+  // d <= 16: the extra (cached Dist) rows start at ring row 16 and rows d..15
+  // stay zero, so that a lane loads all 16 coordinate rows unconditionally
+  const int row0 = DR == 16 ? 16 : d;
+  const Pipe R = pipe_of(L, smraw, row0 + k);
   float* med_s = SMP(float, med);
   ActSlot* act_s = SMP(ActSlot, act);
   int* row_s = SMP(int, row);
@@ -2563,6 +2593,11 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
   for (int j = threadIdx.x; j < d; j += blockDim.x) scale_s[j] = p.scale[j];
   for (int e = threadIdx.x; e < (DR == 16 ? nw : 1) * ncap; e += blockDim.x) acc_s[e] = 0;
   for (int e = threadIdx.x; e < nw * KMAX; e += blockDim.x) cnt_s[e] = 0;
+  if (DR == 16 && d < 16)  // zero padding rows d..15 of every stage (never copied into)
+    for (int e = threadIdx.x; e < p.stages * (16 - d) * R.ldr; e += blockDim.x) {
+      const int sg = e / ((16 - d) * R.ldr), r = e - sg * (16 - d) * R.ldr;
+      R.buf[(size_t)sg * R.rows * R.ldr + (size_t)d * R.ldr + r] = 0.f;
+    }
   pipe_init(p, R, nw);
   __syncthreads();
   if (ctl_s[0]) return;
@@ -2575,10 +2610,16 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
     const unsigned b = __ballot_sync(0xffffffffu, cached);
     const int r = __popc(b & ((1u << a) - 1u));
     if (w == 0) {
-      if (a < na) row_s[a] = cached ? (d + r) * R.ldr : -1;
+      if (a < na) {
+        row_s[a] = cached ? (row0 + r) * R.ldr : -1;
+        ex->drow[a] = p.dist + (size_t)act_s[a].key * p.n_pad;
+      }
     } else {
       if (cached) ex->src[r] = p.dist + (size_t)act_s[a].key * p.n_pad;
-      if (a == 0) ex->n = __popc(b);
+      if (a == 0) {
+        ex->n = __popc(b);
+        ex->row0 = row0;
+      }
       __syncwarp();
     }
   }
@@ -2604,11 +2645,11 @@ __global__ void __launch_bounds__(288, LOC_MINB) k_locality(RunParams p) {
       pipe_produce(p, R, nmy, nullptr, ex);
     } else if constexpr (DR == 16) {
       if (p.metric == 1)
-        loc16_consume<1>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s,
+        loc16_consume<1>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s, ex,
                          L.tab + w * 32 * LOC16_PPT, acc_s + (size_t)w * ncap, cnt_s + w * KMAX, scale_s,
                          nfb);
       else
-        loc16_consume<0>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s,
+        loc16_consume<0>(p, R, L.buf / 4, nmy, na, ncomp, med_s, medd_s, row_s, thr_s, act_s, ex,
                          L.tab + w * 32 * LOC16_PPT, acc_s + (size_t)w * ncap, cnt_s + w * KMAX, scale_s,
                          nfb);
     } else {
@@ -3961,7 +4002,7 @@ PassShape pass_shape(int d, int k, int l, int nM, int num_sms) {
     L.full = b.take(8 * SMAX);
     L.empty = b.take(8 * SMAX);
     // >= 16 rows: k_locality<16> loads rows 0..15 of every stage unconditionally
-    L.buf = b.take((size_t)stages * std::max(d + k, 16) * L.ldr * 4);
+    L.buf = b.take((size_t)stages * ((d <= 16 ? 16 : d) + k) * L.ldr * 4);
     L.med = b.take(4 * (size_t)k * (d < 32 ? 32 : d));  // rows padded to 16 / 32
     L.act = b.take(sizeof(ActSlot) * KMAX);
     L.row = b.take(4 * KMAX);
