@@ -350,7 +350,7 @@ static proclus_status upload_data(proclus_handle* h, const float* data, bool syn
     src = h->staging.p;
   }
   CK(cudaMemsetAsync(h->flag.p, 0, sizeof(int), h->stream));
-  CK(cudaMemsetAsync(h->colmax.p, 0, sizeof(unsigned) * h->d, h->stream));
+  CK(cudaMemsetAsync(h->colmax.p, 0, sizeof(unsigned) * PACK_COPIES * h->d, h->stream));
   launch(h, K_PACK, -1, [&] {
     launch_pack_soa(src, h->n, h->d, h->n_pad, h->xs.p, h->flag.p, h->colmax.p, h->stream);
   });
@@ -478,7 +478,7 @@ proclus_status proclus_create_ex(const float* data, int64_t n, int32_t d,
   }
   if (h->xs.ensure((size_t)h->n_pad * d) != cudaSuccess || h->flag.ensure(1) != cudaSuccess ||
       h->qflag.ensure(1) != cudaSuccess ||
-      h->colmax.ensure((size_t)d) != cudaSuccess || h->scale.ensure((size_t)d) != cudaSuccess ||
+      h->colmax.ensure((size_t)PACK_COPIES * d) != cudaSuccess || h->scale.ensure((size_t)d) != cudaSuccess ||
       h->iscale.ensure((size_t)d) != cudaSuccess)
     return cleanup(
         fail(PROCLUS_ENOMEM, "device allocation of %lld x %d failed", (long long)n, d));

@@ -102,58 +102,121 @@ __device__ __forceinline__ void fence_mbar_init() {
 // ===================================================================== N0
 // row-major [n][d] -> SoA [d][n_pad] (zero padding), non-finite flag and the
 // per-dimension max |x| (as float bits; non-negative floats order as uints).
-// 32 x 32 tiles through shared memory; a block transposes PACK_TILES tiles of
-// consecutive points so that max |x_j| is reduced in the block first (one
-// atomicMax per column per block: the per-thread atomics on d addresses
-// serialised the whole pack).
-constexpr int PACK_TILES = 8;
-__global__ void k_pack_soa(const float* __restrict__ in, long long n, int d,
-                           long long n_pad, float* __restrict__ xs, int* bad,
-                           unsigned* colmax) {
-  __shared__ float tile[32][33];
-  __shared__ float red[8][33];
-  const int j0 = blockIdx.y * 32;
-  const int tx = threadIdx.x, ty = threadIdx.y;
-  int nonfinite = 0;
-  float amax = 0.f;
-  for (int tt = 0; tt < PACK_TILES; ++tt) {
-    const long long p0 = ((long long)blockIdx.x * PACK_TILES + tt) * 32;
-    if (p0 >= n_pad) break;
-    for (int r = ty; r < 32; r += 8) {
-      const long long p = p0 + r;
-      const int j = j0 + tx;
-      float v = 0.f;
-      if (p < n && j < d) {
-        v = in[p * d + j];
-        if (!isfinite(v))
-          nonfinite = 1;
-        else
-          amax = fmaxf(amax, fabsf(v));
+// A block packs pp consecutive points (<= 512, a multiple of 32, <= 48 KB of
+// shared memory): their pp x d floats are one
+// contiguous range of the input, read with coalesced 16-byte loads into
+// shared memory (point q's row at stride ds = d | 1: odd, so the column reads
+// below are conflict-free), then written as d coalesced rows of PK_P floats;
+// max |x_j| is reduced per warp (a warp's 32 consecutive outputs share j),
+// then per block, one atomicMax per column and block.
+constexpr int PK_T = 256;
+__global__ void __launch_bounds__(PK_T) k_pack_soa(const float* __restrict__ in, long long n, int d,
+                                                   long long n_pad, float* __restrict__ xs, int* bad,
+                                                   unsigned* colmax, int PK_P) {
+  extern __shared__ __align__(16) float pk[];  // [pp][ds]
+  const int ds = d | 1;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const long long p0 = (long long)blockIdx.x * PK_P;
+  const int np = (int)(p0 < n ? (n - p0 < PK_P ? n - p0 : PK_P) : 0);
+  const int nf = np * d;
+  const float* src = in + p0 * d;
+  const bool vec = ((reinterpret_cast<unsigned long long>(src) & 15ull) == 0);
+  int e0 = 0;
+  if (vec) {
+    const float4* s4 = reinterpret_cast<const float4*>(src);
+    const int n4 = nf >> 2;
+    if (ds == d) {  // odd d: the shared rows are the input's flat layout: one bulk copy
+      __shared__ __align__(8) unsigned long long pbar;
+      const unsigned bytes = (unsigned)nf * 4u & ~15u;
+      if (tid == 0) {
+        mbar_init(&pbar, 1);
+        fence_mbar_init();
+        if (bytes) {
+          mbar_expect_tx(&pbar, bytes);
+          bulk_g2s(pk, src, bytes, &pbar);
+        }
       }
-      tile[r][tx] = v;
+      for (int f = (int)(bytes >> 2) + tid; f < nf; f += PK_T) pk[f] = src[f];
+      __syncthreads();  // the barrier's init is visible
+      if (bytes) mbar_wait(&pbar, 0u);
+      e0 = nf;
+    } else {  // (q, j) of element 4 e, advanced without division
+      const int step = 4 * PK_T, dq = step / d, dj = step - dq * d;
+      int q = (4 * tid) / d, j = 4 * tid - q * d;
+      for (int e = tid; e < n4; e += PK_T) {
+        const float4 v = __ldcs(s4 + e);
+        const float vv[4] = {v.x, v.y, v.z, v.w};
+        int qq = q, jj = j;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          pk[qq * ds + jj] = vv[c];
+          if (++jj == d) {
+            jj = 0;
+            ++qq;
+          }
+        }
+        q += dq;
+        j += dj;
+        if (j >= d) {
+          j -= d;
+          ++q;
+        }
+      }
     }
-    __syncthreads();
-    for (int r = ty; r < 32; r += 8) {
-      const int j = j0 + r;
-      const long long p = p0 + tx;
-      if (j < d && p < n_pad) xs[(long long)j * n_pad + p] = tile[tx][r];
+    if (ds != d) e0 = n4 << 2;
+  }
+  for (int f = e0 + tid; f < nf; f += PK_T) {
+    const int q = f / d, j = f - q * d;
+    pk[q * ds + j] = __ldcs(src + f);
+  }
+  __syncthreads();
+  // one warp per output row j: consecutive lanes take consecutive points
+  // (coalesced stores; column reads at the odd stride ds are conflict-free)
+  int nonfinite = 0;
+  const int nstore = (int)(n_pad - p0 < PK_P ? n_pad - p0 : PK_P);  // multiple of 32
+  for (int j = w; j < d; j += PK_T / 32) {
+    float amax = 0.f;
+    float* dst = xs + (size_t)j * n_pad + p0;
+    for (int q0 = 0; q0 < nstore; q0 += 128) {
+      float v[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const int q = q0 + 32 * c + lane;
+        v[c] = q < np ? pk[q * ds + j] : 0.f;
+        const float a = fabsf(v[c]);
+        nonfinite |= !(a <= 3.402823466e38f);
+        amax = fmaxf(amax, a);  // a NaN operand is ignored
+      }
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+        if (q0 + 32 * c < nstore) dst[q0 + 32 * c + lane] = v[c];
     }
-    __syncthreads();
+    const unsigned m = __reduce_max_sync(0xffffffffu, __float_as_uint(amax));
+    // one of PACK_COPIES partial maxima per column (same-address atomics
+    // from every block serialised in L2), folded by k_fold_colmax
+    if (lane == 0 && m) atomicMax(colmax + (size_t)(blockIdx.x % PACK_COPIES) * d + j, m);
   }
   if (nonfinite) atomicOr(bad, 1);
-  red[ty][tx] = amax;
-  __syncthreads();
-  if (ty == 0) {
-    float m = red[0][tx];
-    for (int r = 1; r < 8; ++r) m = fmaxf(m, red[r][tx]);
-    if (j0 + tx < d && m > 0.f) atomicMax(colmax + j0 + tx, __float_as_uint(m));
+}
+
+__global__ void k_fold_colmax(unsigned* colmax, int d) {
+  for (int j = threadIdx.x; j < d; j += blockDim.x) {
+    unsigned m = colmax[j];
+    for (int c = 1; c < PACK_COPIES; ++c) m = max(m, colmax[(size_t)c * d + j]);
+    colmax[j] = m;
   }
 }
 
 void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
                      unsigned* colmax, cudaStream_t s) {
-  dim3 grid((unsigned)((n_pad + 32 * PACK_TILES - 1) / (32 * PACK_TILES)), (unsigned)((d + 31) / 32));
-  k_pack_soa<<<grid, dim3(32, 8), 0, s>>>(in, n, d, n_pad, xs, bad, colmax);
+  const int ds = d | 1;
+  int pp = (int)((48 * 1024 / 4) / ds) / 32 * 32;
+  if (pp > 512) pp = 512;
+  if (pp < 32) pp = 32;  // d <= 256 (binding cap): 32 x 257 floats fit
+  const size_t smem = sizeof(float) * (size_t)pp * ds;
+  const unsigned grid = (unsigned)((n_pad + pp - 1) / pp);
+  k_pack_soa<<<grid, PK_T, smem, s>>>(in, n, d, n_pad, xs, bad, colmax, pp);
+  k_fold_colmax<<<1, 256, 0, s>>>(colmax, d);
 }
 
 // Per-dimension fixed-point scales 2^e_j from max |x_j| (colmax, float bits):

@@ -33,7 +33,9 @@ struct PassShape {
 };
 
 // N0: row-major [n][d] -> SoA [d][n_pad]; *bad |= 1 on a non-finite value;
-// colmax[j] = max(colmax[j], bits of max |x_j|).
+// colmax[j] = max(colmax[j], bits of max |x_j|).  colmax holds PACK_COPIES x d
+// words, all zero on entry; copies 1.. are scratch (partial maxima).
+constexpr int PACK_COPIES = 32;
 void launch_pack_soa(const float* in, long long n, int d, long long n_pad, float* xs, int* bad,
                      unsigned* colmax, cudaStream_t s);
 // 2^e_j, 2^-e_j and the quant_sum fma flag from max |x_j| on the device
