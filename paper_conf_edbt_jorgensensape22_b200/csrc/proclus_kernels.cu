@@ -3838,7 +3838,7 @@ __global__ void __launch_bounds__(288) k_cost1(RunParams p) {
 // --- Final AssignPoints with D* (Alg 1 l.18) and RemoveOutliers (l.19):
 // outlier iff seg_{D*_i}(x, m_i) > Delta_i for every i (reading R17).
 template <int PPT>
-__global__ void __launch_bounds__(160) k_final(RunParams p) {
+__global__ void __launch_bounds__(160, 4) k_final(RunParams p) {
   DevState* st = p.st;
   extern __shared__ __align__(16) unsigned char smraw[];
   const SmemLayout& L = p.lay[KK_FIN];
@@ -3877,9 +3877,121 @@ __global__ void __launch_bounds__(160) k_final(RunParams p) {
   int ndmax = 0;
   for (int i = 0; i < k; ++i) ndmax = max(ndmax, nD_s[i]);
   const double G = (double)(ndmax + 6) * 5.9604644775390625e-08;
+  // PPT == 2: clusters in groups of equal |D_c| (as k_assign) and fp32
+  // certified thresholds of the outlier test seg <= Delta_c, rounded outwards
+  __shared__ int ord_s[KMAX], gst_s[KMAX + 1], gnd_s[KMAX], ngrp_s;
+  __shared__ float din_s[KMAX], dout_s[KMAX];
+  if (PPT == 2 && threadIdx.x < 32) {
+    const int c = lane;
+    const int nd = c < k ? nD_s[c] : 1 << 30;
+    int rank = 0;
+    for (int o = 0; o < k; ++o) {
+      const int no = nD_s[o];
+      rank += (no < nd) | ((no == nd) & (o < c));
+    }
+    if (c < k) {
+      ord_s[rank] = c;
+      const double D = Dl_s[c];
+      const bool ok = D >= 1e-30 && D < 1e30;
+      din_s[c] = ok ? __double2float_rd(D * (1.0 - G)) : -1.0f;
+      dout_s[c] = ok ? __double2float_ru(D * (1.0 + G)) : CUDART_INF_F;
+    }
+    __syncwarp();
+    const int r = lane;
+    const int ndr = r < k ? nD_s[ord_s[r]] : -1;
+    const int ndp = __shfl_up_sync(0xffffffffu, ndr, 1);
+    const bool head = r < k && (r == 0 || ndp != ndr);
+    const unsigned hb = __ballot_sync(0xffffffffu, head);
+    if (head) {
+      const int g = __popc(hb & ((1u << lane) - 1u));
+      gst_s[g] = r;
+      gnd_s[g] = ndr;
+    }
+    if (lane == 0) {
+      ngrp_s = __popc(hb);
+      gst_s[__popc(hb)] = k;
+    }
+  }
+  __syncthreads();
   long long nfb = 0;
   if (w == nw) {
     pipe_produce(p, R, nmy, nullptr, nullptr);
+  } else if constexpr (PPT == 2) {
+    // a lane owns the adjacent points q0 + 2 lane + u (packed terms)
+    const int q0 = w * 64, ngrp = ngrp_s;
+    RingPos rp;
+    for (long long i = 0; i < nmy; ++i, rp.next(p.stages)) {
+      const int stg = rp.stg;
+      const long long base = (blockIdx.x + i * gridDim.x) * (long long)P;
+      mbar_wait(R.full_a + 8u * stg, rp.ph);
+      const float* xs = R.buf + (size_t)stg * R.rows * P;
+      const float* xq = xs + q0 + 2 * lane;
+      float best[2], second[2];
+      int bi[2], out[2], und[2];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        best[u] = CUDART_INF_F;
+        second[u] = CUDART_INF_F;
+        bi[u] = 0;
+        out[u] = 1;  // outside every sphere so far (certainly)
+        und[u] = 0;  // some sphere test needs the exact value
+      }
+#define FIN_UPD(c, s)                                                      \
+  do {                                                                     \
+    const float r_ = rcp_s[c], in_ = din_s[c], ou_ = dout_s[c];            \
+    _Pragma("unroll") for (int u = 0; u < 2; ++u) {                        \
+      const float qv = (s)[u] * r_;                                        \
+      second[u] = qv < best[u] ? best[u] : fminf(second[u], qv);           \
+      bi[u] = qv < best[u] ? (c) : bi[u];                                  \
+      best[u] = fminf(best[u], qv);                                        \
+      const bool rng = qv >= 1e-30f && qv < 1e30f;                         \
+      if (rng && qv < in_) out[u] = 0;                                     \
+      else if (!(rng && qv > ou_)) und[u] = 1;                             \
+    }                                                                      \
+  } while (0)
+      for (int g = 0; g < ngrp; ++g) {
+        const int r0 = gst_s[g], r1 = gst_s[g + 1];
+        switch (gnd_s[g]) {
+#define DT(N)                                              \
+  case N:                                                  \
+    for (int r = r0; r < r1; ++r) {                        \
+      const int c = ord_s[r];                              \
+      float s[2];                                          \
+      dist_terms2<N>(xq, tab_s + c * d, s);                \
+      FIN_UPD(c, s);                                       \
+    }                                                      \
+    break;
+          DT(1) DT(2) DT(3) DT(4) DT(5) DT(6) DT(7) DT(8)
+          DT(9) DT(10) DT(11) DT(12) DT(13) DT(14) DT(15) DT(16)
+#undef DT
+          default:
+            for (int r = r0; r < r1; ++r) {
+              const int c = ord_s[r];
+              float s[2];
+              dist_terms2_n(xq, tab_s + c * d, gnd_s[g], s);
+              FIN_UPD(c, s);
+            }
+        }
+      }
+#undef FIN_UPD
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int q = q0 + 2 * lane + u;
+        const long long gp = base + q;
+        if (gp >= p.n) continue;
+        const double b = (double)best[u], s2v = (double)second[u];
+        const bool certain = (b >= 1e-30) && (s2v < 1e30) && (s2v * (1.0 - G) > b * (1.0 + G));
+        int lbl = bi[u], o = out[u];
+        if (!certain || (o && und[u])) {
+          int outx = 0;
+          lbl = exact_argmin(xs + q, P, med_s, dl_s, nD_s, k, d, Dl_s, &outx);
+          if (o && und[u]) o = outx;
+          ++nfb;
+        }
+        p.out_labels[gp] = o ? -1 : lbl;
+      }
+      pipe_release(R, stg);
+    }
   } else {
     const int q0 = w * 32 * PPT;
     RingPos rp;

@@ -16,7 +16,7 @@ for r in $(seq 1 $R); do
 import json,sys
 j=json.loads(open(sys.argv[1]).read().strip().splitlines()[-1])
 k=j["kernels"]
-print(f"{sys.argv[2]:10s} {j['value']:8.1f}/s  loc {k['locality']['us_per_launch']:6.2f}  asg {k['assign']['us_per_launch']:6.2f}  cost {k['cost']['us_per_launch']:6.2f}  tails {j['tails_ms_total']}")
+print(f"{sys.argv[2]:10s} {j['value']:8.1f}/s  loc {k['locality']['us_per_launch']:6.2f}  asg {k['assign']['us_per_launch']:6.2f}  cost {k['cost']['us_per_launch']:6.2f}  fin {k['final']['us_per_launch']:6.2f}  ref {k['refine_x']['us_per_launch']:6.2f}  greedy {k['greedy']['us_per_launch']:6.2f}  tails {j['tails_ms_total']}")
 PY
   done
 done
