@@ -236,6 +236,37 @@ def test_run_multi_levels(pk, orc):
             assert_parity(g, o, what=f"multi level {level} setting {i}")
 
 
+@pytest.mark.parametrize("level", [1, 2, 3])
+def test_run_multi_sweep_extent(pk, orc, level):
+    """The C5 sweep's extremes (BASELINE configs[4]: k up to 20, l up to 10,
+    #M = B k_max = 200) on C2-sized data: every setting of a 3 x 3 grid equals
+    the oracle's multi-parameter run at each reuse level."""
+    data, _ = synth.config_data("C2", seed=3)
+    ks, ls = [5, 12, 20], [3, 6, 10]
+    with pk.Proclus(data) as h:
+        got = h.run_multi(ks, ls, seed=11, reuse_level=level)
+    want = orc.proclus_multi(data, ks, ls, seed=11, reuse_level=level)
+    assert len(got) == len(want) == 9
+    for i, (g, o) in enumerate(zip(got, want)):
+        assert g.medoids.shape[0] == ks[i // 3]
+        assert_parity(g, o, what=f"sweep level {level} (k, l) = ({ks[i // 3]}, {ls[i % 3]})")
+
+
+def test_run_list_full_size_C5_corners(pk, orc):
+    """C5 itself (n = 1M, d = 15) at the corners of its grid, level 2 through
+    run_list with k_sample = 20 (the settings-parallel split of section
+    8(e)): each setting equals the oracle's level-2 sweep over the same
+    corners (S and M drawn once for k_max = 20)."""
+    data, _ = synth.config_data("C3", seed=1)
+    ks, ls = [5, 20], [3, 10]
+    settings = [(k, l) for k in ks for l in ls]
+    with pk.Proclus(data) as h:
+        got = h.run_list(settings, k_sample=20, seed=5, reuse_level=2)
+    want = orc.proclus_multi(data, ks, ls, seed=5, reuse_level=2)
+    for (k, l), g, o in zip(settings, got, want):
+        assert_parity(g, o, what=f"C5 corner (k, l) = ({k}, {l})")
+
+
 # ---------------------------------------------------------------- full sizes
 @pytest.mark.parametrize("metric", [0, 1])
 @pytest.mark.parametrize("name,seed", [("C3", 1), ("C4", 1)])
