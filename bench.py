@@ -579,14 +579,22 @@ def run_sweep(args):
         barrier()
     total_ms = sum(ms)
     launches = lc[0]
-    # level 0: this rank's settings as independent runs (one step)
+    # level 0: this rank's settings as independent runs (one step); every
+    # variant is run once untimed first, as the level-2 sweep was (warm-up),
+    # so that each is timed with its CUDA graphs already instantiated
     indep = lambda s: [h.run(k, l, seed=args.seed0 + s) for k, l in mine]
+    lev1 = lambda s: h.run_list(mine, k_sample=kmax, seed=args.seed0 + s, reuse_level=1)
+    lev3 = lambda s: h.run_multi(ks_grid, ls_grid, seed=args.seed0 + s, reuse_level=3)
+    if args.warmup > 0:
+        indep(2000)
+        lev1(2000)
+        if world == 1:
+            lev3(2000)
     ms0 = timed(indep, 1)
-    ms1 = timed(lambda s: h.run_list(mine, k_sample=kmax, seed=args.seed0 + s, reuse_level=1), 1)
+    ms1 = timed(lev1, 1)
     # level 3: warm start from the previous MBest -- changes results,
     # sequential over the whole grid (one GPU only)
-    ms3 = (timed(lambda s: h.run_multi(ks_grid, ls_grid, seed=args.seed0 + s, reuse_level=3), 1)
-           if world == 1 else [float("nan")])
+    ms3 = timed(lev3, 1) if world == 1 else [float("nan")]
     if world > 1:
         t = torch.tensor([total_ms, ms0[0], ms1[0]], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)

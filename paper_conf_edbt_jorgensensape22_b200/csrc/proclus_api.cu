@@ -183,10 +183,18 @@ struct proclus_handle {
   unsigned char* h_pin = nullptr;
   size_t h_pin_bytes = 0;
   // graph of one run (prepare -> while{loc, asg, cost} -> refine, final)
-  cudaGraphExec_t gexec = nullptr;
-  RunParams gkey;
-  PassShape gshape;
-  bool gvalid = false;
+  // instantiated graphs by (RunParams, PassShape): a multi-parameter sweep
+  // builds one per (k, l) setting (~0.7 ms of host capture + instantiation
+  // with the GPU idle) and later sweeps of the same handle reuse them
+  struct GraphEntry {
+    RunParams key;
+    PassShape shape;
+    cudaGraphExec_t exec;
+    unsigned long long used;
+  };
+  std::vector<GraphEntry> graphs;
+  unsigned long long graph_tick = 0;
+  cudaGraphExec_t gexec = nullptr;  // the graph of the current run (owned by graphs)
   // trace
   int tr_cap = 0;
   DBuf<int> t_mcur;
@@ -529,7 +537,9 @@ void proclus_destroy(proclus_handle* h) {
     cudaEventDestroy(h->pf_done);
     cudaEventDestroy(h->pack_done);
   }
-  if (h->gexec) cudaGraphExecDestroy(h->gexec);
+  for (auto& ge : h->graphs) cudaGraphExecDestroy(ge.exec);
+  h->graphs.clear();
+  h->gexec = nullptr;
   h->xs.release();
   h->staging.release();
   h->flag.release();
@@ -701,14 +711,21 @@ static proclus_status split_tail(proclus_handle* h, const RunParams& p, int tail
 // refine_x -> final.  The cost tail sets the condition.  Rebuilt only when
 // the kernel parameters change (new buffers or setting).
 static proclus_status build_graph(proclus_handle* h, RunParams p, const PassShape& ps) {
-  if (h->gvalid && memcmp(&h->gkey, &p, sizeof(RunParams)) == 0 &&
-      memcmp(&h->gshape, &ps, sizeof(PassShape)) == 0)
-    return PROCLUS_OK;
-  if (h->gexec) {
-    cudaGraphExecDestroy(h->gexec);
-    h->gexec = nullptr;
+  for (auto& ge : h->graphs)
+    if (memcmp(&ge.key, &p, sizeof(RunParams)) == 0 && memcmp(&ge.shape, &ps, sizeof(PassShape)) == 0) {
+      ge.used = ++h->graph_tick;
+      h->gexec = ge.exec;
+      return PROCLUS_OK;
+    }
+  constexpr size_t kMaxGraphs = 256;  // the C5 grid has 128 settings
+  if (h->graphs.size() >= kMaxGraphs) {  // evict the least recently used
+    size_t lru = 0;
+    for (size_t i = 1; i < h->graphs.size(); ++i)
+      if (h->graphs[i].used < h->graphs[lru].used) lru = i;
+    cudaGraphExecDestroy(h->graphs[lru].exec);
+    h->graphs.erase(h->graphs.begin() + (long)lru);
   }
-  h->gvalid = false;
+  h->gexec = nullptr;
   const RunParams key = p;
   cudaGraph_t g;
   CK(cudaGraphCreate(&g, 0));
@@ -752,12 +769,12 @@ static proclus_status build_graph(proclus_handle* h, RunParams p, const PassShap
   launch_final(p, ps, cs);
   CK(cudaStreamEndCapture(cs, &tmp));
   CK(cudaStreamDestroy(cs));
-  cudaError_t e = cudaGraphInstantiate(&h->gexec, g, 0);
+  cudaGraphExec_t ge = nullptr;
+  cudaError_t e = cudaGraphInstantiate(&ge, g, 0);
   cudaGraphDestroy(g);
   CK(e);
-  h->gkey = key;
-  h->gshape = ps;
-  h->gvalid = true;
+  h->graphs.push_back({key, ps, ge, ++h->graph_tick});
+  h->gexec = ge;
   return PROCLUS_OK;
 }
 
