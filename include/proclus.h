@@ -18,8 +18,12 @@
  *    next call on the same thread).
  *  - Input data is row-major (point-major) n x d fp32.  Values must be finite.
  *  - A handle owns all device memory it allocates (data copy, the Dist cache
- *    of P:153, H of eq 5, labels, partial sums).  It is not thread-safe: one
- *    call at a time per handle.  Distinct handles are independent.
+ *    of P:153, H of eq 5, labels, partial sums) and the CUDA graphs it
+ *    instantiates for its runs (one per distinct run shape -- k, l, variant,
+ *    output placement --, at most 256, least recently used evicted; a later
+ *    run of the same shape, e.g. the next sweep over the same (k, l) grid,
+ *    reuses them).  It is not thread-safe: one call at a time per handle.
+ *    Distinct handles are independent.
  *  - Determinism: identical (data, parameters, seed, device type) give
  *    bit-identical outputs.
  *  - Randomness (P:241 leaves it unspecified) follows reading R2: SplitMix64

@@ -5,7 +5,7 @@ TAG=${1:-fin}
 OUT=gpurun_out/$TAG; mkdir -p $OUT
 timeout 2400 python -m pytest tests -m gpu -q -rs > $OUT/tests.log 2>&1; tail -2 $OUT/tests.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 2>&1; tail -1 $OUT/smoke.log
-if [ -z "${NO_SAN:-}" ]; then bash tools/sanitize.sh $TAG/san > /dev/null 2>&1; cat $OUT/san/summary.txt; fi
+if [ -n "${SAN:-}" ]; then bash tools/sanitize.sh $TAG/san > /dev/null 2>&1; cat $OUT/san/summary.txt; fi
 timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err
 timeout 600 python bench.py --impl reference > $OUT/ref.json 2> $OUT/ref.err
 timeout 600 python bench.py --config C4 --steps 20 --no-e2e --no-other-metric > $OUT/c4.json 2> $OUT/c4.err
