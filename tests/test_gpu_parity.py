@@ -154,6 +154,41 @@ def test_load_replaces_data(pk, orc):
     assert_parity(g, orc.proclus(d2, 5, 3, seed=1), what="after load")
 
 
+def test_graph_cache_interleaved_settings(pk, orc):
+    """Runs of different (k, l) alternate on one handle, so the second run of
+    each setting launches the CUDA graph instantiated by its first run: the
+    results are those of the first run and of the oracle."""
+    data, _ = synth.config_data("C2", seed=5)
+    with pk.Proclus(data) as h:
+        first = [h.run(k, l, seed=2) for k, l in ((10, 5), (6, 3), (12, 7))]
+        again = [h.run(k, l, seed=2) for k, l in ((10, 5), (6, 3), (12, 7))]
+    for (k, l), a, b in zip(((10, 5), (6, 3), (12, 7)), first, again):
+        assert np.array_equal(a.labels, b.labels) and np.array_equal(a.dims, b.dims)
+        assert a.cost == b.cost and a.iterations == b.iterations
+        assert_parity(b, orc.proclus(data, k, l, seed=2), what=f"graph cache ({k}, {l})")
+
+
+@pytest.mark.parametrize("d", [15, 16])
+def test_pack_unaligned_ragged_input(pk, orc, d):
+    """k_pack_soa on device-resident input whose base is not 16-byte aligned
+    (scalar load path) and whose n is not a multiple of the pack block
+    (ragged last block), for an odd d (flat shared rows) and an even d
+    (padded rows); also the aligned host-input path of the same data."""
+    import torch
+
+    data = synth.generate(3001, d, 5, 3, seed=21)
+    buf = torch.empty(data.size + 1, dtype=torch.float32, device="cuda")
+    view = buf[1:].view(data.shape)  # base offset 4 bytes
+    view.copy_(torch.from_numpy(data))
+    assert view.data_ptr() % 16 != 0
+    with pk.Proclus(view) as h:
+        g = h.run(5, 3, seed=4)
+    with pk.Proclus(data) as h:
+        g2 = h.run(5, 3, seed=4)
+    assert np.array_equal(g.labels, g2.labels) and g.cost == g2.cost
+    assert_parity(g, orc.proclus(data, 5, 3, seed=4), what=f"unaligned input d={d}")
+
+
 @pytest.mark.parametrize("seed", [1, 2, 3])
 def test_run_multi_level3_grids(pk, orc, seed):
     """Level 3 over a grid where k grows and shrinks, and a repeated
