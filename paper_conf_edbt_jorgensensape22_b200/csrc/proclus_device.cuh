@@ -14,7 +14,6 @@ constexpr int WMAX = 8;     // warps per pass block
 constexpr int UMAX = 4;     // points per thread in a chunk
 constexpr int SMAX = 3;     // max bulk-copy ring depth
 constexpr int NCOPY = 8;    // copies of the global accumulators (atomic spread)
-constexpr int DREG = 32;    // d <= DREG: a point's coordinates live in registers
 constexpr int PAD_ALIGN = 1024;  // n_pad multiple; shard boundaries for invariance
 
 // One medoid slot whose locality set changes in this iteration

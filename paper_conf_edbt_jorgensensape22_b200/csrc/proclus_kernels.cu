@@ -1274,12 +1274,6 @@ __device__ __forceinline__ void warp_cells(const float* __restrict__ xs, int P, 
   }
 }
 
-// Publish one warp-uniform ballot per (set, u) for the cells of this warp.
-__device__ __forceinline__ void put_ballot(unsigned* bal, int idx, bool pred) {
-  const unsigned b = __ballot_sync(0xffffffffu, pred);
-  if ((threadIdx.x & 31) == 0) bal[idx] = b;
-}
-
 // ============================================================ smem carving
 struct Carve {
   char* ptr;
@@ -1326,39 +1320,6 @@ __device__ __forceinline__ int cert_le(float f, double T, double G) {
   if (fd < T * (1.0 - G)) return 1;
   if (fd > T * (1.0 + G)) return 0;
   return -1;
-}
-
-// fp32 approximation of the full-space distance of one staged point (stride P).
-__device__ __forceinline__ float approx_full(const float* __restrict__ x, int P,
-                                             const float* __restrict__ m, int d, int metric) {
-  float s = 0.f;
-  if (metric == 1) {
-    for (int j = 0; j < d; ++j) s += fabsf(x[j * P] - m[j]);
-    return s;
-  }
-  for (int j = 0; j < d; ++j) {
-    const float t = x[j * P] - m[j];
-    s = fmaf(t, t, s);
-  }
-  return sqrtf(s);
-}
-// same with the point in registers (d <= DREG)
-__device__ __forceinline__ float approx_full_reg(const float (&x)[DREG],
-                                                 const float* __restrict__ m, int d, int metric) {
-  float s = 0.f;
-  if (metric == 1) {
-#pragma unroll
-    for (int j = 0; j < DREG; ++j)
-      if (j < d) s += fabsf(x[j] - m[j]);
-    return s;
-  }
-#pragma unroll
-  for (int j = 0; j < DREG; ++j)
-    if (j < d) {
-      const float t = x[j] - m[j];
-      s = fmaf(t, t, s);
-    }
-  return sqrtf(s);
 }
 
 // Exact (oracle) argmin of seg_{D_i}(x, m_i) = (sum_{j in D_i} |x_j - m_ij|)/|D_i|
@@ -2798,7 +2759,7 @@ __device__ __forceinline__ float hi_f(unsigned long long v) {
 
 // Paired-point terms (assign, 2 points per lane at xp, xp + 1): one 64-bit
 // shared load and one packed subtraction per term serve both points; the
-// two sums are formed in the same order as dist_terms<2, ND>.
+// two sums are formed in two chains (even / odd terms).
 template <int ND>
 __device__ __forceinline__ void dist_terms2(const float* __restrict__ xp,
                                             const Term* __restrict__ tb, float (&s)[2]) {
@@ -2842,64 +2803,6 @@ __device__ __noinline__ void dist_terms2_n(const float* __restrict__ xp,
   s[1] = a1 + b1;
 }
 
-// Segmental distance terms of one cluster for PPT points: fp32 partial sums
-// in two chains (the certified bound only needs the number of terms, DESIGN.md
-// section 5).  ND is the compile-time |D_i| (fully unrolled); the _n variant
-// handles |D_i| > 16.
-template <int PPT, int ND>
-__device__ __forceinline__ void dist_terms(const float* __restrict__ xq,
-                                           const Term* __restrict__ tb, float (&s)[PPT]) {
-  float a[PPT], b[PPT];
-#pragma unroll
-  for (int u = 0; u < PPT; ++u) {
-    a[u] = 0.f;
-    b[u] = 0.f;
-  }
-#pragma unroll
-  for (int t = 0; t < ND; t += 2) {
-    const Term e0 = tb[t];
-    if (t + 1 < ND) {
-      const Term e1 = tb[t + 1];
-#pragma unroll
-      for (int u = 0; u < PPT; ++u) {
-        a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
-        b[u] += fabsf(LDX(xq + u * 32, e1.joff) - e1.m);
-      }
-    } else {
-#pragma unroll
-      for (int u = 0; u < PPT; ++u) a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
-    }
-  }
-#pragma unroll
-  for (int u = 0; u < PPT; ++u) s[u] = ND > 1 ? a[u] + b[u] : a[u];
-}
-
-template <int PPT>
-__device__ __noinline__ void dist_terms_n(const float* __restrict__ xq, const Term* __restrict__ tb,
-                                          int nd, float (&s)[PPT]) {
-  float a[PPT], b[PPT];
-#pragma unroll
-  for (int u = 0; u < PPT; ++u) {
-    a[u] = 0.f;
-    b[u] = 0.f;
-  }
-  int t = 0;
-  for (; t + 2 <= nd; t += 2) {
-    const Term e0 = tb[t], e1 = tb[t + 1];
-#pragma unroll
-    for (int u = 0; u < PPT; ++u) {
-      a[u] += fabsf(LDX(xq + u * 32, e0.joff) - e0.m);
-      b[u] += fabsf(LDX(xq + u * 32, e1.joff) - e1.m);
-    }
-  }
-  if (t < nd) {
-    const Term e = tb[t];
-#pragma unroll
-    for (int u = 0; u < PPT; ++u) a[u] += fabsf(LDX(xq + u * 32, e.joff) - e.m);
-  }
-#pragma unroll
-  for (int u = 0; u < PPT; ++u) s[u] = a[u] + b[u];
-}
 
 // --- AssignPoints (Alg 5) + centroid sums for long rows (chunks of P <= 64
 // points): the ASW_NW consumer warps share every chunk instead of owning 32
@@ -3483,7 +3386,8 @@ __device__ __forceinline__ void pipe_init_k(const SmemLayout& L, const Pipe& R) 
 // --- AssignPoints (Alg 5) + centroid sums of EvaluateCluster (Alg 6 l.1-8),
 // chunks of >= 128 points.  A lane owns the adjacent points q0 + 2 lane + u
 // (u = 0, 1) of its warp's 64 columns: certified fp32 argmin over the
-// clusters (packed terms, one switch per cluster on the warp-uniform |D_c|),
+// clusters (packed terms; clusters visited in groups of equal |D_c|, one
+// switch per group selects the unrolled term code),
 // fp64 fallback near a tie (reading R8), u8 label.  Then the chunk is
 // counting-sorted by the new labels among the consumer threads and the item
 // threads (cell (c, t), residue r, stride R_c ~ |C_c|) add round(x_j 2^e_j)
