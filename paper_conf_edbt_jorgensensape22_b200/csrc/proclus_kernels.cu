@@ -2780,6 +2780,71 @@ __device__ __forceinline__ void dist_terms2(const float* __restrict__ xp,
   s[0] = ND > 1 ? a0 + b0 : a0;
   s[1] = ND > 1 ? a1 + b1 : a1;
 }
+// The same with 32-bit shared-window addresses (xa: the lane's first point
+// in a ring stage, ta: the cluster's first table entry), so that no 64-bit
+// generic pointers stay live across the cluster loop.
+__device__ __forceinline__ void lds_term(unsigned a, unsigned long long& m2, int& joff) {
+  unsigned lo, hi, jo;
+  asm volatile("{\n.reg .b32 pad;\nld.shared.v4.b32 {%0, %1, %2, pad}, [%3];\n}"
+               : "=r"(lo), "=r"(hi), "=r"(jo)
+               : "r"(a));
+  m2 = ((unsigned long long)hi << 32) | lo;
+  joff = (int)jo;
+}
+__device__ __forceinline__ unsigned long long lds_u64(unsigned a) {
+  unsigned long long v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
+  return v;
+}
+template <int ND>
+__device__ __forceinline__ void dist_terms2s(unsigned xa, unsigned ta, float (&s)[2]) {
+  float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+#pragma unroll
+  for (int t = 0; t < ND; t += 2) {
+    unsigned long long m0;
+    int j0;
+    lds_term(ta + 16u * t, m0, j0);
+    const unsigned long long r0 = fsub2(lds_u64(xa + (unsigned)j0), m0);
+    a0 += fabsf(lo_f(r0));
+    a1 += fabsf(hi_f(r0));
+    if (t + 1 < ND) {
+      unsigned long long m1;
+      int j1;
+      lds_term(ta + 16u * (t + 1), m1, j1);
+      const unsigned long long r1 = fsub2(lds_u64(xa + (unsigned)j1), m1);
+      b0 += fabsf(lo_f(r1));
+      b1 += fabsf(hi_f(r1));
+    }
+  }
+  s[0] = ND > 1 ? a0 + b0 : a0;
+  s[1] = ND > 1 ? a1 + b1 : a1;
+}
+__device__ __noinline__ void dist_terms2s_n(unsigned xa, unsigned ta, int nd, float (&s)[2]) {
+  float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
+  int t = 0;
+  for (; t + 2 <= nd; t += 2) {
+    unsigned long long m0, m1;
+    int j0, j1;
+    lds_term(ta + 16u * t, m0, j0);
+    lds_term(ta + 16u * (t + 1), m1, j1);
+    const unsigned long long r0 = fsub2(lds_u64(xa + (unsigned)j0), m0);
+    const unsigned long long r1 = fsub2(lds_u64(xa + (unsigned)j1), m1);
+    a0 += fabsf(lo_f(r0));
+    a1 += fabsf(hi_f(r0));
+    b0 += fabsf(lo_f(r1));
+    b1 += fabsf(hi_f(r1));
+  }
+  if (t < nd) {
+    unsigned long long m;
+    int j;
+    lds_term(ta + 16u * t, m, j);
+    const unsigned long long r = fsub2(lds_u64(xa + (unsigned)j), m);
+    a0 += fabsf(lo_f(r));
+    a1 += fabsf(hi_f(r));
+  }
+  s[0] = a0 + b0;
+  s[1] = a1 + b1;
+}
 __device__ __noinline__ void dist_terms2_n(const float* __restrict__ xp,
                                            const Term* __restrict__ tb, int nd, float (&s)[2]) {
   float a0 = 0.f, a1 = 0.f, b0 = 0.f, b1 = 0.f;
@@ -3504,6 +3569,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
       mbar_wait(R.full_a + 8u * stg, rp.ph);
       const float* xs = R.buf + (size_t)stg * R.rows * P;
       const float* xq = xs + q0 + 2 * lane;
+      const unsigned xqa = smem_u32(xq), taa = smem_u32(tab_s);
       float best[2], second[2];
       int bi[2];
 #pragma unroll
@@ -3522,7 +3588,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
     for (int r = r0; r < r1; ++r) {                        \
       const int c = ord_s[r];                              \
       float s[2];                                          \
-      dist_terms2<N>(xq, tab_s + c * d, s);                \
+      dist_terms2s<N>(xqa, taa + 16u * (unsigned)(c * d), s); \
       ASG_UPD(c, s);                                       \
     }                                                      \
     break;
@@ -3533,7 +3599,7 @@ __global__ void __launch_bounds__(160) k_assign(RunParams p) {
             for (int r = r0; r < r1; ++r) {
               const int c = ord_s[r];
               float s[2];
-              dist_terms2_n(xq, tab_s + c * d, gnd_s[g], s);
+              dist_terms2s_n(xqa, taa + 16u * (unsigned)(c * d), gnd_s[g], s);
               ASG_UPD(c, s);
             }
         }
