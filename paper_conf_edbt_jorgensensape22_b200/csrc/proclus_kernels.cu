@@ -357,7 +357,10 @@ __device__ __forceinline__ unsigned long long dkey(double v);
 // receiver's mbarrier; a CTA proceeds when all CS*GC_W = 32 candidates landed
 // and reduces them with one warp argmax (slots parity double buffered: pick
 // i uses slot i&1).
-constexpr int GC_TPB = 64;
+#ifndef GC_CS
+#define GC_CS 8  // CTAs per greedy cluster (32 warps in all; 8 x 128 threads: 58 vs 60 us at C3)
+#endif
+constexpr int GC_TPB = 1024 / GC_CS;  // threads per CTA
 constexpr int GC_W = GC_TPB / 32;
 
 __device__ __forceinline__ unsigned cluster_rank() {
@@ -806,7 +809,7 @@ static cudaError_t greedy_smem_launch(const float* srows, int nS, int d, int nM,
 template <int NP, int METRIC, int DP>
 static cudaError_t greedy_cluster_launch(const double* sT, int nS, int d, int dp, int nM, int q0,
                                          int* spos, double* pickdist, cudaStream_t s) {
-  constexpr int CS = 16;
+  constexpr int CS = GC_CS;
   const size_t bytes = sizeof(double) * (size_t)NP * CS * GC_TPB * dp;
   auto fn = k_greedy_cluster<NP, METRIC, CS, DP>;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
@@ -921,7 +924,7 @@ template <int NP>
 __global__ void __launch_bounds__(GC_TPB)
     k_greedy_mat(const double* __restrict__ Ds, int nS, int nM, int q0, int* __restrict__ spos,
                  double* __restrict__ pickdist) {
-  constexpr int CS = 16;
+  constexpr int CS = GC_CS;
   static_assert(CS * GC_W == 32, "one candidate slot per lane");
   __shared__ __align__(16) unsigned cand[2][CS * GC_W][4];
   __shared__ __align__(8) unsigned long long bar[2];
@@ -993,7 +996,7 @@ __global__ void __launch_bounds__(GC_TPB)
 template <int NP>
 static cudaError_t greedy_mat_launch(const double* Ds, int nS, int nM, int q0, int* spos,
                                      double* pickdist, cudaStream_t s) {
-  constexpr int CS = 16;
+  constexpr int CS = GC_CS;
   auto fn = k_greedy_mat<NP>;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   if (e != cudaSuccess) return e;
@@ -1015,7 +1018,7 @@ static cudaError_t greedy_mat_launch(const double* Ds, int nS, int nM, int q0, i
 cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int metric,
                           double* scratch, int* spos, double* pickdist, cudaStream_t s) {
   {  // cluster of 16 CTAs x 64 threads: NP positions per thread
-    const int per = 16 * GC_TPB;
+    const int per = GC_CS * GC_TPB;
     const int npc = nS <= per ? 1 : nS <= 2 * per ? 2 : nS <= 4 * per ? 4 : 0;
     const int dp = d <= 8 ? 8 : d <= 16 ? 16 : d <= 32 ? 32 : ((d + 1) / 2) * 2;
     const size_t soa = (size_t)dp * npc * per;  // doubles
@@ -1039,7 +1042,7 @@ cudaError_t launch_greedy(const float* srows, int nS, int d, int nM, int q0, int
   if (nS <= GM_PPT * GM_TPB) {  // <= 4096: exact matrix, picks in a 16-CTA cluster
     const int nt = (nS + SD_T - 1) / SD_T;
     k_sdist_tiled<<<nt * (nt + 1) / 2, 256, 0, s>>>(srows, nS, d, metric, scratch);
-    const int per = 16 * GC_TPB;
+    const int per = GC_CS * GC_TPB;
     return nS <= 2 * per ? greedy_mat_launch<2>(scratch, nS, nM, q0, spos, pickdist, s)
                          : greedy_mat_launch<4>(scratch, nS, nM, q0, spos, pickdist, s);
   }
