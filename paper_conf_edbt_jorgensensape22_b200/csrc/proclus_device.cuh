@@ -13,7 +13,11 @@ constexpr int TPB_MAX = 1024;  // threads of the standalone tail kernels
 constexpr int WMAX = 8;     // warps per pass block
 constexpr int UMAX = 4;     // points per thread in a chunk
 constexpr int SMAX = 3;     // max bulk-copy ring depth
-constexpr int NCOPY = 8;    // copies of the global accumulators (atomic spread)
+#ifndef PROCLUS_NCOPY
+#define PROCLUS_NCOPY 2
+#endif
+constexpr int NCOPY = PROCLUS_NCOPY;  // copies of the global accumulators (atomic spread; 2: the
+                                      // tails load fewer copies, 1 serialises the cost flush)
 constexpr int PAD_ALIGN = 1024;  // n_pad multiple; shard boundaries for invariance
 
 // One medoid slot whose locality set changes in this iteration
