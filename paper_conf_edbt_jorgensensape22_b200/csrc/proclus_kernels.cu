@@ -59,6 +59,16 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phas
       "r"(phase)
       : "memory");
 }
+#ifndef MBAR_HINT_NS
+#define MBAR_HINT_NS 10000000  // suspend-time hint (ns) of the ring waits; 0: none
+#endif
+#define PC_STR_(x) #x
+#define PC_STR(x) PC_STR_(x)
+#if MBAR_HINT_NS > 0
+#define MBAR_HINT ", " PC_STR(MBAR_HINT_NS)
+#else
+#define MBAR_HINT ""
+#endif
 // the same with the barrier's 32-bit shared address computed once per kernel
 // (a generic-to-shared conversion per spin iteration costs an S2UR chain)
 __device__ __forceinline__ void mbar_wait(unsigned bar, unsigned phase) {
@@ -66,7 +76,7 @@ __device__ __forceinline__ void mbar_wait(unsigned bar, unsigned phase) {
       "{\n"
       ".reg .pred p;\n"
       "WAITA_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 0x989680;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1" MBAR_HINT ";\n"
       "@!p bra WAITA_%=;\n"
       "}\n" ::"r"(bar),
       "r"(phase)
